@@ -1,0 +1,176 @@
+/*
+ * spgemm.h — C ABI of the B200-native (sm_100a) hash-based two-phase CSR SpGEMM
+ *            C = A * B  (Nagasaka, Nukada, Matsuoka, ICPP 2017; /root/reference/PAPER.md).
+ *
+ * Library: paper_conf_icpp_nagasakanm17_b200/libspgemm.so.  extern "C", plain pointers and
+ * sizes only; no CUDA or torch types appear in a signature (streams are passed as the
+ * opaque value of a cudaStream_t, `void*`).  Pointers are DEVICE pointers unless marked
+ * (host).
+ *
+ * Problem statement: A (m x k) and B (k x n) and C are CSR; the
+ * pattern of C is unknown until computed, so a counting ("symbolic") pass sizes C exactly
+ * before a calculation ("numeric") pass fills it — the two-pass strategy of PAPER.md:68
+ * that "does not require redundant working memory".
+ *
+ * CSR layout: row i of X is col[rpt[i] .. rpt[i+1]) with values at the same
+ * offsets.  rpt is int64 (nnz(C) exceeds 2^31 at R-MAT scale 22 — DESIGN.md reading R17),
+ * col is int32, 0 <= col < n <= 2^31-2 (the key -1 is the empty-slot marker of
+ * Algorithm 5).  a_rpt[0] need NOT be 0 (zero-copy row slices).
+ * Input rows need not be sorted; duplicate column indices behave as their sum.  Explicit
+ * zeros and cancellations are kept structurally (reading R6).  Output rows are sorted by
+ * ascending column.
+ *
+ * Ownership: the caller owns A, B and all of C.  The library owns only its workspace
+ * (grouping arrays, n_prod, global-memory hash tables), obtained from the allocator given to
+ * spgemm_create (NULL -> cudaMallocAsync on the handle's stream).  A's and B's structure
+ * arrays are BORROWED from spgemm_symbolic until the next spgemm_symbolic/destroy: they
+ * must stay alive and unchanged while spgemm_numeric may be called (structure reuse).
+ *
+ * Ordering: all work is enqueued on the handle's stream (plus internal streams forked from
+ * and joined back into it).  spgemm_symbolic returns after synchronising that stream (the
+ * host needs nnz(C) to allocate C — PAPER.md:80, 282).  spgemm_numeric is asynchronous.
+ * A handle is not thread-safe: one handle per host thread / stream.
+ *
+ * Errors: status codes only; no C++ exception crosses the ABI.  Detailed text via
+ * spgemm_last_error(h).  Any CUDA failure returns SPGEMM_ERR_CUDA.
+ */
+#ifndef SPGEMM_H_
+#define SPGEMM_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SPGEMM_API __attribute__((visibility("default")))
+#else
+#define SPGEMM_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct spgemm_ctx *spgemm_handle_t;
+
+typedef enum { SPGEMM_F32 = 0, SPGEMM_F64 = 1 } spgemm_dtype_t;
+
+typedef enum {
+    SPGEMM_OK = 0,
+    SPGEMM_ERR_INVALID_ARG = 1,     /* NULL pointer, negative size, bad enum */
+    SPGEMM_ERR_BAD_STATE = 2,       /* numeric before symbolic, etc. */
+    SPGEMM_ERR_OOM = 3,             /* allocator returned NULL */
+    SPGEMM_ERR_CUDA = 4,            /* CUDA runtime error; text in spgemm_last_error */
+    SPGEMM_ERR_INDEX_OVERFLOW = 5,  /* n > 2^31-2 or m >= 2^31 */
+    SPGEMM_ERR_NOT_SUPPORTED = 6,   /* device is not sm_100 */
+    SPGEMM_ERR_INVALID_INPUT = 7    /* validation on: rpt not monotone or col out of range */
+} spgemm_status_t;
+
+/* Stream-ordered allocator callbacks.  alloc returns NULL on failure. */
+typedef struct {
+    void *(*alloc)(size_t bytes, void *stream, void *ctx);
+    void (*free)(void *ptr, size_t bytes, void *stream, void *ctx);
+    void *ctx;
+} spgemm_allocator_t;
+
+/* Create a handle on CUDA device `device`, enqueueing on `stream` (a cudaStream_t; NULL =
+ * legacy default stream).  alloc may be NULL.  Fails with NOT_SUPPORTED off sm_100. */
+SPGEMM_API spgemm_status_t spgemm_create(spgemm_handle_t *h, int device, void *stream,
+                              const spgemm_allocator_t *alloc);
+
+/* Phase 1, steps (1)-(4) of PAPER.md:80 (Figure 1):
+ *   (1) n_prod per row (Algorithm 2),
+ *   (2) grouping of rows by n_prod (Table I, B200 table),
+ *   (3) per-group hash counting of each row's distinct columns (Algorithms 3-5,
+ *       PAPER.md:98-155) with the shared-memory -> global-memory overflow retry of
+ *       PAPER.md:155, 181,
+ *   (4) prefix sum into c_rpt, plus step (6) grouping by nnz for phase 2.
+ * m, k, n: shapes of A (m x k) and B (k x n).  a_rpt: m+1, a_col: a_rpt[m]-a_rpt[0] used
+ * entries (indexed by a_rpt values).  b_rpt: k+1, b_col.  c_rpt: m+1 int64, caller-
+ * allocated, filled with c_rpt[0] = 0.  c_nnz (host): exact nnz(C).  nprod (host,
+ * nullable): sum of intermediate products (the FLOPS numerator / 2).
+ * Synchronises the handle's stream before returning. */
+SPGEMM_API spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t n,
+                                const int64_t *a_rpt, const int32_t *a_col,
+                                const int64_t *b_rpt, const int32_t *b_col,
+                                int64_t *c_rpt, int64_t *c_nnz, int64_t *nprod);
+
+/* Phase 2, step (7) of PAPER.md:80 and §III-C: per-group hash
+ * accumulation of values, gather of the non-empty entries and sort by column, written to
+ * c_col / c_val (exactly c_nnz elements each, caller-allocated).  a_val / b_val: values of
+ * the A and B given to the last spgemm_symbolic, both of dtype `dt`; accumulation is in
+ * that working precision.  Asynchronous on the handle's stream; may be
+ * called repeatedly after one symbolic (new values, same structure). */
+SPGEMM_API spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt,
+                               const void *a_val, const void *b_val,
+                               int32_t *c_col, void *c_val);
+
+/* Release the handle and all library workspace. */
+SPGEMM_API spgemm_status_t spgemm_destroy(spgemm_handle_t h);
+
+SPGEMM_API const char *spgemm_status_string(spgemm_status_t s);
+SPGEMM_API const char *spgemm_last_error(spgemm_handle_t h); /* owned by h; valid until next call */
+
+/* ---------------------------------------------------------------- tuning / inspection */
+
+typedef enum {
+    SPGEMM_OPT_SYM_MIN_GROUP = 0,   /* force every row into group >= v (-1 = off); the
+                                       last group index = global-memory fallback */
+    SPGEMM_OPT_NUM_MIN_GROUP = 1,   /* same for the numeric grouping */
+    SPGEMM_OPT_SYM_FILL_LIMIT = 2,  /* optimistic shared-memory table: abort a row after v
+                                       distinct keys (default table/2) */
+    SPGEMM_OPT_STREAMS = 3,         /* 1 = one stream per group, 0 = serial */
+    SPGEMM_OPT_VALIDATE = 4,        /* 1 = O(nnz) input validation in spgemm_symbolic */
+    SPGEMM_OPT_LANES = 5,           /* lanes per B row (power of two 1..32), 0 = auto */
+    SPGEMM_OPT_WORKSPACE_BUDGET = 6,/* max bytes for global-memory hash tables */
+    SPGEMM_OPT_TIMING = 7           /* 1 = per-group CUDA-event timing (default 1) */
+} spgemm_option_t;
+
+SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);
+
+#define SPGEMM_MAX_GROUPS 16
+
+/* Counters of the last symbolic/numeric call.  Times are CUDA-event milliseconds measured on
+ * the stream each kernel was launched on (group kernels: their own stream). */
+typedef struct {
+    int64_t m, k, n, nnz_a, nnz_b, nnz_c, nprod;
+    int64_t max_row_nprod, max_row_nnz;
+    int32_t n_sym_groups, n_num_groups;
+    int64_t sym_rows[SPGEMM_MAX_GROUPS], num_rows[SPGEMM_MAX_GROUPS];
+    int64_t sym_nprod[SPGEMM_MAX_GROUPS], num_nprod[SPGEMM_MAX_GROUPS];
+    int64_t sym_nnza[SPGEMM_MAX_GROUPS], num_nnza[SPGEMM_MAX_GROUPS];
+    int64_t num_nnzc[SPGEMM_MAX_GROUPS];
+    int64_t sym_overflow_rows;          /* rows retried in the global-memory table */
+    float sym_group_ms[SPGEMM_MAX_GROUPS], num_group_ms[SPGEMM_MAX_GROUPS];
+    float setup_ms, symbolic_ms, scan_ms, numeric_ms; /* phases (Figure 5/6 breakdown) */
+    int64_t kernel_launches_symbolic, kernel_launches_numeric;
+    int64_t workspace_bytes, workspace_peak_bytes;
+} spgemm_stats_t;
+
+SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);
+
+/* Group table of the implementation: inclusive upper bounds of each group's key (n_prod
+ * for phase 1, nnz for phase 2), ascending; the group after the last bound is the global-
+ * memory fallback.  *ngroups (host) receives the number of bounds. */
+SPGEMM_API spgemm_status_t spgemm_group_bounds(int phase /* 1 or 2 */, int64_t *upper /* host, >= 16 */,
+                                    int32_t *ngroups /* host */);
+
+/* Copy the per-row n_prod (int64, m) and the grouping permutation of `phase` (int32, m:
+ * row ids concatenated group by group) plus group offsets (int64, ngroups+2) of the last
+ * symbolic call to HOST buffers (for tests). */
+SPGEMM_API spgemm_status_t spgemm_get_grouping(spgemm_handle_t h, int phase, int64_t *nprod,
+                                    int32_t *perm, int64_t *offsets);
+
+/* Multi-GPU row partition: n_prod-balanced contiguous row blocks of A for nparts ranks.
+ * splits (host, nparts+1): splits[0] = 0, splits[nparts] = m, and block p holds rows
+ * [splits[p], splits[p+1]) with prefix(n_prod) crossing p*total/nparts at its start. */
+SPGEMM_API spgemm_status_t spgemm_row_partition(spgemm_handle_t h, int64_t m, int64_t k,
+                                     const int64_t *a_rpt, const int32_t *a_col,
+                                     const int64_t *b_rpt, int32_t nparts, int64_t *splits);
+
+/* Library build info, e.g. "spgemm sm_100a <date>" (static string). */
+SPGEMM_API const char *spgemm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPGEMM_H_ */

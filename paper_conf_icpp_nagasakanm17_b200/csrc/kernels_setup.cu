@@ -1,0 +1,336 @@
+// kernels_setup.cu — steps (1), (2), (4), (6) of PAPER.md:80 (Figure 1) on sm_100a:
+//   k_nprod_group   Alg. 2 fused with the step-(2) group id + per-group
+//                   histogram, CTA-aggregated before the global atomics.
+//   k_group_scatter "the grouping is done by generating the array of gathered row indices
+//                   corresponding to each group": warp-aggregated (MATCH.ANY)
+//                   CTA-local ranks, one global atomic per group per CTA.
+//   k_scan_*        step (4): inclusive prefix sum of nnz_i into rpt_C (3-kernel tile scan),
+//                   the first kernel fused with the step-(6) grouping by nnz_i.
+//   k_validate      optional O(nnz) input validation.
+//   k_splits        n_prod-balanced row blocks for the multi-GPU driver.
+#include "spgemm_internal.cuh"
+
+namespace spg {
+
+namespace {
+
+constexpr int kSetupThreads = 256;
+
+__device__ __forceinline__ int group_of(long long key, const Bounds& bd) {
+  int g = 0;
+  while (g < bd.nbounds && key > bd.upper[g]) ++g;
+  if (g < bd.min_group) g = bd.min_group;
+  return g;
+}
+
+template <int LPR>
+__global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
+    long long m, const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
+    const int64_t* __restrict__ b_rpt, int64_t* __restrict__ nprod, uint8_t* __restrict__ grp,
+    int64_t* __restrict__ c_rpt, DevAcc* __restrict__ acc, Bounds bd) {
+  __shared__ unsigned long long s_rows[kMaxGroups], s_np[kMaxGroups], s_nza[kMaxGroups];
+  __shared__ unsigned long long s_total, s_max;
+  if (threadIdx.x < kMaxGroups) {
+    s_rows[threadIdx.x] = 0; s_np[threadIdx.x] = 0; s_nza[threadIdx.x] = 0;
+  }
+  if (threadIdx.x == 0) { s_total = 0; s_max = 0; }
+  __syncthreads();
+  constexpr int RPB = kSetupThreads / LPR;
+  const long long row = (long long)blockIdx.x * RPB + threadIdx.x / LPR;
+  const int l = threadIdx.x % LPR;
+  long long np = 0, a0 = 0, a1 = 0;
+  if (row < m) {
+    a0 = a_rpt[row];
+    a1 = a_rpt[row + 1];
+    // Alg. 2: n_prod += rpt_B[col_A[j]+1] - rpt_B[col_A[j]], j in [rpt_A[i], rpt_A[i+1])
+    for (long long j = a0 + l; j < a1; j += LPR) {
+      const int kk = __ldg(a_col + j);
+      np += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
+    }
+  }
+#pragma unroll
+  for (int off = LPR / 2; off > 0; off >>= 1) np += __shfl_xor_sync(0xffffffffu, np, off);
+  if (row < m && l == 0) {
+    nprod[row] = np;
+    int g = 0xFF;
+    if (np == 0) {
+      c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
+    } else {
+      g = group_of(np, bd);
+      atomicAdd(&s_rows[g], 1ull);
+      atomicAdd(&s_np[g], (unsigned long long)np);
+      atomicAdd(&s_nza[g], (unsigned long long)(a1 - a0));
+    }
+    grp[row] = (uint8_t)g;
+    atomicAdd(&s_total, (unsigned long long)np);
+    atomicMax(&s_max, (unsigned long long)np);
+  }
+  __syncthreads();
+  if (threadIdx.x < kMaxGroups && s_rows[threadIdx.x]) {
+    atomicAdd(&acc->sym_rows[threadIdx.x], s_rows[threadIdx.x]);
+    atomicAdd(&acc->sym_nprod[threadIdx.x], s_np[threadIdx.x]);
+    atomicAdd(&acc->sym_nnza[threadIdx.x], s_nza[threadIdx.x]);
+  }
+  if (threadIdx.x == 0) {
+    atomicAdd(&acc->total_nprod, s_total);
+    atomicMax(&acc->max_nprod, s_max);
+  }
+}
+
+constexpr int kScatterItems = 4;
+
+__global__ __launch_bounds__(kSetupThreads) void k_group_scatter(long long m, const uint8_t* __restrict__ grp,
+                                                                 Offsets off, int* __restrict__ cursor,
+                                                                 int32_t* __restrict__ perm) {
+  __shared__ int s_cnt[kMaxGroups], s_base[kMaxGroups];
+  if (threadIdx.x < kMaxGroups) s_cnt[threadIdx.x] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  int g[kScatterItems], local[kScatterItems];
+  long long rowv[kScatterItems];
+#pragma unroll
+  for (int it = 0; it < kScatterItems; ++it) {
+    const long long row = ((long long)blockIdx.x * kScatterItems + it) * kSetupThreads + threadIdx.x;
+    rowv[it] = row;
+    g[it] = row < m ? grp[row] : 0xFF;
+    const unsigned peers = __match_any_sync(0xffffffffu, g[it]);
+    const int leader = __ffs(peers) - 1;
+    const int rank = __popc(peers & ((1u << lane) - 1u));
+    int base = 0;
+    if (lane == leader && g[it] != 0xFF) base = atomicAdd(&s_cnt[g[it]], __popc(peers));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    local[it] = base + rank;
+  }
+  __syncthreads();
+  if (threadIdx.x < off.ngroups && s_cnt[threadIdx.x])
+    s_base[threadIdx.x] = atomicAdd(&cursor[threadIdx.x], s_cnt[threadIdx.x]);
+  __syncthreads();
+#pragma unroll
+  for (int it = 0; it < kScatterItems; ++it)
+    if (g[it] != 0xFF) perm[off.off[g[it]] + s_base[g[it]] + local[it]] = (int32_t)rowv[it];
+}
+
+// ------------------------------------------------------------------ scan (+ step-6 grouping)
+constexpr int kScanItems = 8;
+constexpr int kScanTile = kSetupThreads * kScanItems;
+
+__device__ __forceinline__ long long block_sum_ll(long long v, long long* ws) {
+  return Grp<kSetupThreads>::sum(v, ws);
+}
+
+// Tile reduction of x[0..m) (x = rpt_C + 1 holding nnz_i), fused with grouping by nnz_i.
+__global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(
+    long long m, const int64_t* __restrict__ x, long long* __restrict__ tile_sums,
+    const int64_t* __restrict__ nprod, const int64_t* __restrict__ a_rpt, uint8_t* __restrict__ grp2,
+    DevAcc* __restrict__ acc, Bounds bd) {
+  __shared__ long long ws[33];
+  __shared__ unsigned long long s_rows[kMaxGroups], s_np[kMaxGroups], s_nza[kMaxGroups], s_nzc[kMaxGroups];
+  __shared__ unsigned long long s_max;
+  const bool grouping = grp2 != nullptr;
+  if (grouping) {
+    if (threadIdx.x < kMaxGroups) {
+      s_rows[threadIdx.x] = 0; s_np[threadIdx.x] = 0; s_nza[threadIdx.x] = 0; s_nzc[threadIdx.x] = 0;
+    }
+    if (threadIdx.x == 0) s_max = 0;
+    __syncthreads();
+  }
+  const long long base = (long long)blockIdx.x * kScanTile;
+  long long s = 0;
+#pragma unroll
+  for (int e = 0; e < kScanItems; ++e) {
+    const long long i = base + e * kSetupThreads + threadIdx.x;
+    if (i < m) {
+      const long long v = x[i];
+      s += v;
+      if (grouping) {
+        int g = 0xFF;
+        if (v > 0) {
+          g = group_of(v, bd);
+          atomicAdd(&s_rows[g], 1ull);
+          atomicAdd(&s_nzc[g], (unsigned long long)v);
+          atomicAdd(&s_np[g], (unsigned long long)nprod[i]);
+          atomicAdd(&s_nza[g], (unsigned long long)(a_rpt[i + 1] - a_rpt[i]));
+          atomicMax(&s_max, (unsigned long long)v);
+        }
+        grp2[i] = (uint8_t)g;
+      }
+    }
+  }
+  const long long tot = block_sum_ll(s, ws);
+  if (threadIdx.x == 0) tile_sums[blockIdx.x] = tot;
+  if (grouping) {
+    __syncthreads();
+    if (threadIdx.x < kMaxGroups && s_rows[threadIdx.x]) {
+      atomicAdd(&acc->num_rows[threadIdx.x], s_rows[threadIdx.x]);
+      atomicAdd(&acc->num_nnzc[threadIdx.x], s_nzc[threadIdx.x]);
+      atomicAdd(&acc->num_nprod[threadIdx.x], s_np[threadIdx.x]);
+      atomicAdd(&acc->num_nnza[threadIdx.x], s_nza[threadIdx.x]);
+    }
+    if (threadIdx.x == 0) atomicMax(&acc->max_nnz, s_max);
+  }
+}
+
+// Exclusive scan of the tile sums, one CTA of 1024 threads, carried across chunks.
+__global__ __launch_bounds__(1024) void k_scan_tiles(long long ntiles, long long* __restrict__ t) {
+  __shared__ long long ws[33];
+  long long carry = 0;
+  for (long long c = 0; c < ntiles; c += 1024) {
+    const long long i = c + threadIdx.x;
+    const long long v = i < ntiles ? t[i] : 0;
+    long long tot;
+    const long long ex = Grp<1024>::excl_scan(v, &tot, ws);
+    if (i < ntiles) t[i] = carry + ex;
+    carry += tot;
+    __syncthreads();
+  }
+}
+
+// In-place inclusive scan of each tile plus its offset.  Blocked arrangement: thread owns
+// kScanItems consecutive elements.
+__global__ __launch_bounds__(kSetupThreads) void k_scan_down(long long m, int64_t* __restrict__ x,
+                                                             const long long* __restrict__ tile_off,
+                                                             long long* __restrict__ total_out) {
+  __shared__ long long ws[33];
+  const long long base = (long long)blockIdx.x * kScanTile + (long long)threadIdx.x * kScanItems;
+  long long v[kScanItems];
+  long long s = 0;
+#pragma unroll
+  for (int e = 0; e < kScanItems; ++e) {
+    const long long i = base + e;
+    v[e] = i < m ? x[i] : 0;
+    s += v[e];
+  }
+  long long tot;
+  long long run = Grp<kSetupThreads>::excl_scan(s, &tot, ws) + tile_off[blockIdx.x];
+#pragma unroll
+  for (int e = 0; e < kScanItems; ++e) {
+    const long long i = base + e;
+    run += v[e];
+    if (i < m) {
+      x[i] = run;
+      if (i == m - 1 && total_out) *total_out = run;
+    }
+  }
+}
+
+// ------------------------------------------------------------------ validation
+__global__ void k_validate(long long m, long long k, long long n, const int64_t* __restrict__ a_rpt,
+                           const int32_t* __restrict__ a_col, const int64_t* __restrict__ b_rpt,
+                           const int32_t* __restrict__ b_col, int* __restrict__ err) {
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long tid = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  bool bad = false;
+  for (long long i = tid; i < m; i += stride) bad |= a_rpt[i + 1] < a_rpt[i];
+  for (long long i = tid; i < k; i += stride) bad |= b_rpt[i + 1] < b_rpt[i];
+  const long long a0 = a_rpt[0], a1 = a_rpt[m], b0 = b_rpt[0], b1 = b_rpt[k];
+  if (a0 < 0 || b0 < 0) bad = true;
+  for (long long j = a0 + tid; j < a1; j += stride) { const int c = a_col[j]; bad |= (c < 0 || c >= k); }
+  for (long long j = b0 + tid; j < b1; j += stride) { const int c = b_col[j]; bad |= (c < 0 || c >= n); }
+  if (bad) atomicOr(err, 1);
+}
+
+// n_prod only (no grouping) for the partition.
+__global__ __launch_bounds__(kSetupThreads) void k_nprod_only(long long m, const int64_t* __restrict__ a_rpt,
+                                                              const int32_t* __restrict__ a_col,
+                                                              const int64_t* __restrict__ b_rpt,
+                                                              int64_t* __restrict__ out) {
+  const long long row = (long long)blockIdx.x * (kSetupThreads / 32) + threadIdx.x / 32;
+  const int l = threadIdx.x & 31;
+  long long np = 0;
+  if (row < m)
+    for (long long j = a_rpt[row] + l; j < a_rpt[row + 1]; j += 32) {
+      const int kk = a_col[j];
+      np += b_rpt[kk + 1] - b_rpt[kk];
+    }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) np += __shfl_xor_sync(0xffffffffu, np, off);
+  if (row < m && l == 0) out[row] = np;
+}
+
+// splits[p] = min{ r in [0,m] : sum_{i<r} n_prod_i >= p*total/P }, splits[P] = m.
+__global__ void k_splits(long long m, const int64_t* __restrict__ excl, int nparts, int64_t* __restrict__ splits) {
+  const int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p > nparts) return;
+  if (p == nparts) { splits[p] = m; return; }
+  const long long total = excl[m];
+  const long long target = (long long)((__int128)total * p / nparts);
+  long long lo = 0, hi = m;
+  while (lo < hi) {
+    const long long mid = (lo + hi) / 2;
+    if (excl[mid] >= target) hi = mid; else lo = mid + 1;
+  }
+  splits[p] = lo;
+}
+
+}  // namespace
+
+cudaError_t launch_nprod_group(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,
+                               const int64_t* b_rpt, int64_t* nprod, uint8_t* grp, int64_t* c_rpt,
+                               DevAcc* acc, Bounds b, int lpr_log2) {
+  if (m == 0) return cudaSuccess;
+  const int lpr = 1 << lpr_log2;
+  const long long rpb = kSetupThreads / lpr;
+  const unsigned grid = (unsigned)((m + rpb - 1) / rpb);
+  switch (lpr_log2) {
+#define SPG_CASE(L) case L: k_nprod_group<(1 << L)><<<grid, kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod, grp, c_rpt, acc, b); break;
+    SPG_CASE(0) SPG_CASE(1) SPG_CASE(2) SPG_CASE(3) SPG_CASE(4) SPG_CASE(5)
+#undef SPG_CASE
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_group_scatter(cudaStream_t s, long long m, const uint8_t* grp, Offsets off, int* cursor,
+                                 int32_t* perm) {
+  if (m == 0) return cudaSuccess;
+  const long long per = (long long)kSetupThreads * kScatterItems;
+  k_group_scatter<<<(unsigned)((m + per - 1) / per), kSetupThreads, 0, s>>>(m, grp, off, cursor, perm);
+  return cudaGetLastError();
+}
+
+size_t scan_workspace_bytes(long long m) {
+  return (size_t)((m + kScanTile - 1) / kScanTile + 1) * sizeof(long long);
+}
+
+static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const int64_t* nprod,
+                                  const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
+                                  long long* tile_ws, long long* total_out, int* nlaunch) {
+  if (m == 0) return cudaSuccess;
+  const long long ntiles = (m + kScanTile - 1) / kScanTile;
+  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, nprod, a_rpt, grp2, acc, b);
+  k_scan_tiles<<<1, 1024, 0, s>>>(ntiles, tile_ws);
+  k_scan_down<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, total_out);
+  if (nlaunch) *nlaunch += 3;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const int64_t* nprod,
+                                  const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
+                                  long long* tile_ws, int* nlaunch) {
+  return scan_inclusive(s, m, c_rpt + 1, nprod, a_rpt, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
+}
+
+cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
+                            const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int* err) {
+  k_validate<<<1184, 256, 0, s>>>(m, k, n, a_rpt, a_col, b_rpt, b_col, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,
+                             const int64_t* b_rpt, int64_t* nprod_scan, long long* tile_ws, int nparts,
+                             int64_t* splits_dev, int* nlaunch) {
+  cudaError_t e = cudaMemsetAsync(nprod_scan, 0, sizeof(int64_t), s);
+  if (e != cudaSuccess) return e;
+  if (m > 0) {
+    const long long rpb = kSetupThreads / 32;
+    k_nprod_only<<<(unsigned)((m + rpb - 1) / rpb), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod_scan + 1);
+    Bounds none{};
+    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
+    if (e != cudaSuccess) return e;
+  }
+  k_splits<<<(nparts + 1 + 255) / 256, 256, 0, s>>>(m, nprod_scan, nparts, splits_dev);
+  if (nlaunch) *nlaunch += 2;
+  return cudaGetLastError();
+}
+
+}  // namespace spg

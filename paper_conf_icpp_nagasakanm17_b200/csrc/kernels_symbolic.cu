@@ -1,0 +1,150 @@
+// kernels_symbolic.cu — step (3) of PAPER.md:80: count nnz of each row of C with per-row
+// hash tables (§III-B), one kernel per group (Table I, B200 values in
+// spgemm_internal.cuh).
+//
+// Thread assignment (Alg. 3/4) generalised: a row is owned by TPR threads
+// (4..32 lanes = PWARP/ROW family, or a whole CTA = TB/ROW); inside the row, sub-groups of
+// VW = 2^vw_log2 lanes take successive non-zeros of A (Alg. 4's "one warp per a_ik") and
+// stride VW over the B row (Alg. 4's "one thread per b_kj").  VW is chosen from the mean B
+// row length so short B rows (graphs) do not idle 32-lane warps; VW = 1 is exactly Alg. 3.
+//
+// Hash table: Alg. 5 in shared memory (hash_insert), t_size a power of two >= 2x the
+// group's n_prod bound, so it cannot overflow.  The optimistic group (rows above the last
+// bound) uses the largest table and aborts a row once it has found `fill_limit` distinct
+// keys; the row index is recorded and the row is recounted in a global-memory table sized
+// from its n_prod by k_sym_global.
+#include "spgemm_internal.cuh"
+
+namespace spg {
+
+namespace {
+
+template <int T, int TPR, int BS, bool OPT>
+__global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
+  extern __shared__ __align__(16) int smem[];
+  __shared__ long long ws[33];
+  __shared__ int s_cnt, s_abort;
+  constexpr int RPB = BS / TPR;
+  static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
+  const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
+  int* table = smem + g * T;
+  const long long ridx = (long long)blockIdx.x * RPB + g;
+
+  int4* t4 = reinterpret_cast<int4*>(table);
+  for (int s = t; s < T / 4; s += TPR) t4[s] = make_int4(-1, -1, -1, -1);
+  if (OPT && threadIdx.x == 0) { s_cnt = 0; s_abort = 0; }
+  Grp<TPR>::sync();
+
+  int cnt = 0, row = -1;
+  if (ridx < a.nrows) {
+    row = a.rows[ridx];
+    const long long a0 = a.a_rpt[row], a1 = a.a_rpt[row + 1];
+    const int vwl = a.vw_log2;
+    const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = TPR >> vwl;
+    for (long long j = a0 + sub; j < a1; j += nsub) {
+      if (OPT && ld_volatile(&s_abort)) break;
+      const int kk = __ldg(a.a_col + j);
+      const long long b0 = __ldg(a.b_rpt + kk), b1 = __ldg(a.b_rpt + kk + 1);
+      for (long long q = b0 + lane; q < b1; q += vw) {
+        const int key = __ldg(a.b_col + q);
+        if constexpr (OPT) {
+          if (ld_volatile(&s_abort)) break;
+          if (hash_insert(table, T - 1, key) && atomicAdd(&s_cnt, 1) + 1 >= a.fill_limit) s_abort = 1;
+        } else {
+          cnt += hash_insert(table, T - 1, key);
+        }
+      }
+    }
+  }
+  if constexpr (OPT) {
+    __syncthreads();
+    if (threadIdx.x == 0 && row >= 0) {
+      if (s_abort) {
+        const int p = atomicAdd(a.overflow_count, 1);
+        a.overflow_rows[p] = row;  // PAPER.md:155 "records the row index, and immediately terminates"
+      } else {
+        a.c_cnt[row] = s_cnt;
+      }
+    }
+  } else {
+    const long long tot = Grp<TPR>::sum(cnt, ws);
+    if (t == 0 && row >= 0) a.c_cnt[row] = tot;
+  }
+}
+
+// Global-memory table per CTA (slab of slab_T ints), one row at a time; table size
+// next_pow2(2*min(n_prod_i, n)) so load factor <= 1/2 ("enough large hash table
+// on global memory ... set based on the number of intermediate products").
+__global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
+  __shared__ long long ws[33];
+  int* table = a.slab + (long long)blockIdx.x * a.slab_T;
+  const long long nA = a.nrows;
+  const long long nB = a.dev_count ? (long long)*a.dev_count : 0;
+  const int t = threadIdx.x;
+  for (long long i = blockIdx.x; i < nA + nB; i += gridDim.x) {
+    const int row = i < nA ? a.rows[i] : a.overflow_rows[i - nA];
+    long long cap = a.nprod[row] < a.n ? a.nprod[row] : a.n;
+    long long T = 64;
+    while (T < 2 * cap) T <<= 1;
+    if (T > a.slab_T) T = a.slab_T;
+    int4* t4 = reinterpret_cast<int4*>(table);
+    for (long long s = t; s < T / 4; s += 1024) t4[s] = make_int4(-1, -1, -1, -1);
+    __syncthreads();
+    int cnt = 0;
+    const long long a0 = a.a_rpt[row], a1 = a.a_rpt[row + 1];
+    const int vwl = a.vw_log2;
+    const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = 1024 >> vwl;
+    for (long long j = a0 + sub; j < a1; j += nsub) {
+      const int kk = __ldg(a.a_col + j);
+      const long long b0 = __ldg(a.b_rpt + kk), b1 = __ldg(a.b_rpt + kk + 1);
+      for (long long q = b0 + lane; q < b1; q += vw) cnt += hash_insert(table, (unsigned)(T - 1), __ldg(a.b_col + q));
+    }
+    const long long tot = Grp<1024>::sum(cnt, ws);
+    if (t == 0) a.c_cnt[row] = tot;
+    __syncthreads();
+  }
+}
+
+template <int T, int TPR, int BS, bool OPT>
+cudaError_t launch_sym(cudaStream_t s, const SymArgs& a) {
+  constexpr int RPB = BS / TPR;
+  constexpr int smem = RPB * T * 4;
+  static_assert(smem <= kSmemLimit - 1024, "symbolic table too large");
+  static bool configured = false;
+  if (!configured) {
+    cudaError_t e = cudaFuncSetAttribute(k_sym_smem<T, TPR, BS, OPT>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    configured = true;
+  }
+  SymArgs b = a;
+  const int max_vw = TPR < 32 ? TPR : 32;
+  while ((1 << b.vw_log2) > max_vw) --b.vw_log2;
+  const long long grid = (a.nrows + RPB - 1) / RPB;
+  k_sym_smem<T, TPR, BS, OPT><<<(unsigned)grid, BS, smem, s>>>(b);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_symbolic_group(cudaStream_t s, int group, const SymArgs& a, int /*num_sms*/) {
+  if (a.nrows <= 0) return cudaSuccess;
+  switch (group) {
+#define SPG_G(I)                                                                              \
+  case I:                                                                                     \
+    return launch_sym<kSymGroups[I].T, kSymGroups[I].TPR, kSymGroups[I].BS, (I == kSymOptimistic)>(s, a);
+    SPG_G(0) SPG_G(1) SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9) SPG_G(10)
+#undef SPG_G
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_symbolic_global(cudaStream_t s, const SymArgs& a, int grid) {
+  if (grid <= 0) return cudaSuccess;
+  SymArgs b = a;
+  if (b.vw_log2 > 5) b.vw_log2 = 5;
+  k_sym_global<<<grid, 1024, 0, s>>>(b);
+  return cudaGetLastError();
+}
+
+}  // namespace spg

@@ -1,0 +1,661 @@
+// spgemm.cu — C ABI (include/spgemm.h) and host orchestration of the two-phase hash SpGEMM
+// (Figure 1 steps (1)-(7)) on one B200.
+//
+//   spgemm_symbolic:  (1)+(2) k_nprod_group  -> [sync 1: group sizes, max n_prod]
+//                     (2) k_group_scatter
+//                     (3) per-group hash-count kernels, one stream per group,
+//                         optimistic group -> global retry on the same stream
+//                     (4) tile scan into rpt_C, fused with (6)'s grouping by nnz
+//                     -> [sync 2: nnz(C)] (the host must allocate C exactly)
+//   spgemm_numeric:   (6) k_group_scatter by nnz, (7) per-group accumulate/gather/sort kernels,
+//                     one stream per group; asynchronous.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "spgemm.h"
+#include "spgemm_internal.cuh"
+
+using namespace spg;
+
+namespace {
+
+constexpr int kNumStreams = 8;
+
+struct Buf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+long long next_pow2(long long x) {
+  long long p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+}  // namespace
+
+struct spgemm_ctx {
+  int device = 0;
+  int num_sms = 148;
+  cudaStream_t stream = nullptr;
+  spgemm_allocator_t alloc{};
+  bool user_alloc = false;
+  cudaStream_t gs[kNumStreams]{};
+  cudaEvent_t fork_ev = nullptr;
+  cudaEvent_t join_ev[kNumStreams]{};
+  cudaEvent_t ev[8]{};
+  cudaEvent_t gstart[2][kMaxGroups]{}, gstop[2][kMaxGroups]{};
+  bool gtimed[2][kMaxGroups]{};
+  // options
+  int sym_min_group = -1, num_min_group = -1, fill_limit = 0, use_streams = 1, validate = 0, lanes = 0;
+  int timing = 1;
+  long long ws_budget = 8LL << 30;
+  // state of the last symbolic call
+  int state = 0;
+  bool numeric_done = false;
+  long long m = 0, k = 0, n = 0, nnza = 0, nnzb = 0, nnzc = 0;
+  const int64_t *a_rpt = nullptr, *b_rpt = nullptr;
+  const int32_t *a_col = nullptr, *b_col = nullptr;
+  int64_t* c_rpt = nullptr;
+  int vw_log2 = 0;
+  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, slab_sym;
+  bool perm2_ready = false;
+  DevAcc* hacc = nullptr;      // pinned
+  long long* hends = nullptr;  // pinned: a_rpt[0], a_rpt[m], b_rpt[0], b_rpt[k]
+  DevAcc snap1{}, snap2{};
+  spgemm_stats_t stats{};
+  long long ws_cur = 0, ws_peak = 0;
+  std::string err;
+};
+
+namespace {
+
+spgemm_status_t fail(spgemm_handle_t h, spgemm_status_t s, const std::string& msg) {
+  if (h) h->err = msg;
+  return s;
+}
+
+spgemm_status_t fail_cuda(spgemm_handle_t h, cudaError_t e, const char* what) {
+  char buf[512];
+  snprintf(buf, sizeof buf, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+  return fail(h, SPGEMM_ERR_CUDA, buf);
+}
+
+#define CK(x)                                                  \
+  do {                                                         \
+    cudaError_t e_ = (x);                                      \
+    if (e_ != cudaSuccess) return fail_cuda(h, e_, #x);        \
+  } while (0)
+
+spgemm_status_t buf_alloc(spgemm_handle_t h, Buf& b, size_t bytes) {
+  b.p = nullptr;
+  b.bytes = 0;
+  if (bytes == 0) return SPGEMM_OK;
+  bytes = (bytes + 255) & ~size_t(255);
+  if (h->user_alloc) {
+    b.p = h->alloc.alloc(bytes, (void*)h->stream, h->alloc.ctx);
+    if (!b.p) return fail(h, SPGEMM_ERR_OOM, "allocator returned NULL for " + std::to_string(bytes) + " bytes");
+  } else {
+    cudaError_t e = cudaMallocAsync(&b.p, bytes, h->stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      b.p = nullptr;
+      return fail(h, SPGEMM_ERR_OOM, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
+    }
+  }
+  b.bytes = bytes;
+  h->ws_cur += (long long)bytes;
+  h->ws_peak = std::max(h->ws_peak, h->ws_cur);
+  return SPGEMM_OK;
+}
+
+void buf_free(spgemm_handle_t h, Buf& b) {
+  if (!b.p) return;
+  if (h->user_alloc) h->alloc.free(b.p, b.bytes, (void*)h->stream, h->alloc.ctx);
+  else cudaFreeAsync(b.p, h->stream);
+  h->ws_cur -= (long long)b.bytes;
+  b.p = nullptr;
+  b.bytes = 0;
+}
+
+void release_state(spgemm_handle_t h) {
+  Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow, &h->slab_sym};
+  for (Buf* b : all) buf_free(h, *b);
+  h->state = 0;
+  h->perm2_ready = false;
+}
+
+#define ALLOC(buf, bytes)                                          \
+  do {                                                             \
+    spgemm_status_t s_ = buf_alloc(h, (buf), (bytes));             \
+    if (s_ != SPGEMM_OK) return s_;                                \
+  } while (0)
+
+Bounds sym_bounds(int min_group) {
+  Bounds b{};
+  for (int i = 0; i < kNumSymBounds; ++i) b.upper[i] = kSymGroups[i].upper;
+  b.nbounds = kNumSymBounds;
+  b.min_group = min_group;
+  return b;
+}
+
+Bounds num_bounds(int min_group) {
+  Bounds b{};
+  for (int i = 0; i < kNumNumBounds; ++i) b.upper[i] = kNumGroups[i].upper;
+  b.nbounds = kNumNumBounds;
+  b.min_group = min_group;
+  return b;
+}
+
+Offsets offsets_of(const unsigned long long* rows, int ngroups) {
+  Offsets o{};
+  o.ngroups = ngroups;
+  long long run = 0;
+  for (int g = 0; g < ngroups; ++g) {
+    o.off[g] = run;
+    run += (long long)rows[g];
+  }
+  o.off[ngroups] = run;
+  return o;
+}
+
+cudaStream_t group_stream(spgemm_handle_t h, int g) { return h->use_streams ? h->gs[g % kNumStreams] : h->stream; }
+
+cudaError_t fork(spgemm_handle_t h) {
+  if (!h->use_streams) return cudaSuccess;
+  cudaError_t e = cudaEventRecord(h->fork_ev, h->stream);
+  for (int i = 0; i < kNumStreams && e == cudaSuccess; ++i) e = cudaStreamWaitEvent(h->gs[i], h->fork_ev, 0);
+  return e;
+}
+
+cudaError_t join(spgemm_handle_t h) {
+  if (!h->use_streams) return cudaSuccess;
+  cudaError_t e = cudaSuccess;
+  for (int i = 0; i < kNumStreams && e == cudaSuccess; ++i) {
+    e = cudaEventRecord(h->join_ev[i], h->gs[i]);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(h->stream, h->join_ev[i], 0);
+  }
+  return e;
+}
+
+int auto_vw_log2(spgemm_handle_t h) {
+  if (h->lanes > 0) {
+    int l = 0;
+    while ((1 << (l + 1)) <= h->lanes && l < 5) ++l;
+    return l;
+  }
+  const double avg = h->k > 0 ? (double)h->nnzb / (double)h->k : 1.0;
+  int l = 0;
+  while (l < 5 && (double)(1 << (l + 1)) <= avg * 1.5) ++l;
+  return l;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* spgemm_version(void) { return "spgemm-b200 sm_100a (" __DATE__ ")"; }
+
+const char* spgemm_status_string(spgemm_status_t s) {
+  switch (s) {
+    case SPGEMM_OK: return "SPGEMM_OK";
+    case SPGEMM_ERR_INVALID_ARG: return "SPGEMM_ERR_INVALID_ARG";
+    case SPGEMM_ERR_BAD_STATE: return "SPGEMM_ERR_BAD_STATE";
+    case SPGEMM_ERR_OOM: return "SPGEMM_ERR_OOM";
+    case SPGEMM_ERR_CUDA: return "SPGEMM_ERR_CUDA";
+    case SPGEMM_ERR_INDEX_OVERFLOW: return "SPGEMM_ERR_INDEX_OVERFLOW";
+    case SPGEMM_ERR_NOT_SUPPORTED: return "SPGEMM_ERR_NOT_SUPPORTED";
+    case SPGEMM_ERR_INVALID_INPUT: return "SPGEMM_ERR_INVALID_INPUT";
+  }
+  return "SPGEMM_ERR_UNKNOWN";
+}
+
+const char* spgemm_last_error(spgemm_handle_t h) { return h ? h->err.c_str() : "null handle"; }
+
+spgemm_status_t spgemm_group_bounds(int phase, int64_t* upper, int32_t* ngroups) {
+  if (!upper || !ngroups || (phase != 1 && phase != 2)) return SPGEMM_ERR_INVALID_ARG;
+  if (phase == 1) {
+    for (int i = 0; i < kNumSymBounds; ++i) upper[i] = kSymGroups[i].upper;
+    *ngroups = kNumSymBounds;
+  } else {
+    for (int i = 0; i < kNumNumBounds; ++i) upper[i] = kNumGroups[i].upper;
+    *ngroups = kNumNumBounds;
+  }
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_create(spgemm_handle_t* out, int device, void* stream, const spgemm_allocator_t* alloc) {
+  if (!out) return SPGEMM_ERR_INVALID_ARG;
+  *out = nullptr;
+  if (alloc && (!alloc->alloc || !alloc->free)) return SPGEMM_ERR_INVALID_ARG;
+  spgemm_ctx* h = new spgemm_ctx();
+  h->device = device;
+  h->stream = (cudaStream_t)stream;
+  if (alloc) {
+    h->alloc = *alloc;
+    h->user_alloc = true;
+  }
+  cudaDeviceProp prop;
+  cudaError_t e = cudaGetDeviceProperties(&prop, device);
+  if (e != cudaSuccess) {
+    spgemm_status_t s = fail_cuda(h, e, "cudaGetDeviceProperties");
+    *out = h;  // keep the handle so spgemm_last_error works; caller destroys it
+    return s;
+  }
+  if (prop.major != 10) {
+    *out = h;
+    return fail(h, SPGEMM_ERR_NOT_SUPPORTED, std::string("device is not sm_100 (B200): ") + prop.name);
+  }
+  h->num_sms = prop.multiProcessorCount;
+  DeviceGuard g(device);
+  for (int i = 0; i < kNumStreams; ++i) {
+    e = cudaStreamCreateWithFlags(&h->gs[i], cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->join_ev[i], cudaEventDisableTiming);
+    if (e != cudaSuccess) break;
+  }
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->fork_ev, cudaEventDisableTiming);
+  for (int i = 0; i < 8 && e == cudaSuccess; ++i) e = cudaEventCreate(&h->ev[i]);
+  for (int p = 0; p < 2; ++p)
+    for (int i = 0; i < kMaxGroups && e == cudaSuccess; ++i) {
+      e = cudaEventCreate(&h->gstart[p][i]);
+      if (e == cudaSuccess) e = cudaEventCreate(&h->gstop[p][i]);
+    }
+  if (e == cudaSuccess) e = cudaMallocHost(&h->hacc, sizeof(DevAcc));
+  if (e == cudaSuccess) e = cudaMallocHost(&h->hends, 4 * sizeof(long long));
+  *out = h;
+  if (e != cudaSuccess) return fail_cuda(h, e, "spgemm_create");
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_destroy(spgemm_handle_t h) {
+  if (!h) return SPGEMM_ERR_INVALID_ARG;
+  {
+    DeviceGuard g(h->device);
+    if (h->hacc) {  // hacc is allocated only on a supported device
+      release_state(h);
+      cudaStreamSynchronize(h->stream);
+    }
+    for (int i = 0; i < kNumStreams; ++i) {
+      if (h->gs[i]) cudaStreamDestroy(h->gs[i]);
+      if (h->join_ev[i]) cudaEventDestroy(h->join_ev[i]);
+    }
+    if (h->fork_ev) cudaEventDestroy(h->fork_ev);
+    for (auto& e : h->ev) if (e) cudaEventDestroy(e);
+    for (int p = 0; p < 2; ++p)
+      for (int i = 0; i < kMaxGroups; ++i) {
+        if (h->gstart[p][i]) cudaEventDestroy(h->gstart[p][i]);
+        if (h->gstop[p][i]) cudaEventDestroy(h->gstop[p][i]);
+      }
+    if (h->hacc) cudaFreeHost(h->hacc);
+    if (h->hends) cudaFreeHost(h->hends);
+  }
+  delete h;
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t v) {
+  if (!h) return SPGEMM_ERR_INVALID_ARG;
+  switch (opt) {
+    case SPGEMM_OPT_SYM_MIN_GROUP:
+      if (v < -1 || v > kSymGlobal) return fail(h, SPGEMM_ERR_INVALID_ARG, "SYM_MIN_GROUP out of range");
+      h->sym_min_group = (int)v; break;
+    case SPGEMM_OPT_NUM_MIN_GROUP:
+      if (v < -1 || v > kNumGlobal) return fail(h, SPGEMM_ERR_INVALID_ARG, "NUM_MIN_GROUP out of range");
+      h->num_min_group = (int)v; break;
+    case SPGEMM_OPT_SYM_FILL_LIMIT:
+      if (v < 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "FILL_LIMIT < 0");
+      h->fill_limit = (int)std::min<int64_t>(v, 1 << 30); break;
+    case SPGEMM_OPT_STREAMS: h->use_streams = v ? 1 : 0; break;
+    case SPGEMM_OPT_VALIDATE: h->validate = v ? 1 : 0; break;
+    case SPGEMM_OPT_LANES:
+      if (v < 0 || v > 32 || (v & (v - 1))) return fail(h, SPGEMM_ERR_INVALID_ARG, "LANES must be 0 or a power of two <= 32");
+      h->lanes = (int)v; break;
+    case SPGEMM_OPT_WORKSPACE_BUDGET:
+      if (v <= 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "budget must be > 0");
+      h->ws_budget = v; break;
+    case SPGEMM_OPT_TIMING: h->timing = v ? 1 : 0; break;
+    default: return fail(h, SPGEMM_ERR_INVALID_ARG, "unknown option");
+  }
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t n, const int64_t* a_rpt,
+                                const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col,
+                                int64_t* c_rpt, int64_t* c_nnz, int64_t* nprod_out) {
+  if (!h) return SPGEMM_ERR_INVALID_ARG;
+  if (!h->hacc) return fail(h, SPGEMM_ERR_BAD_STATE, "handle was not created successfully");
+  if (m < 0 || k < 0 || n < 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "negative dimension");
+  if (!a_rpt || !b_rpt || !c_rpt || !c_nnz) return fail(h, SPGEMM_ERR_INVALID_ARG, "NULL pointer argument");
+  if (n > 2147483646LL || m >= 2147483647LL || k >= 2147483647LL)
+    return fail(h, SPGEMM_ERR_INDEX_OVERFLOW, "dimensions exceed int32 column/row indices");
+  DeviceGuard dg(h->device);
+  release_state(h);
+  h->numeric_done = false;
+  h->m = m; h->k = k; h->n = n;
+  h->a_rpt = a_rpt; h->a_col = a_col; h->b_rpt = b_rpt; h->b_col = b_col; h->c_rpt = c_rpt;
+  memset(&h->stats, 0, sizeof h->stats);
+  memset(h->gtimed, 0, sizeof h->gtimed);
+  h->ws_peak = h->ws_cur;
+  h->stats.m = m; h->stats.k = k; h->stats.n = n;
+  h->stats.n_sym_groups = kNumSymGroups;
+  h->stats.n_num_groups = kNumNumGroups;
+  long long launches = 0;
+
+  CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));
+  ALLOC(h->acc, sizeof(DevAcc));
+  CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
+  DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+  if (m == 0) {
+    CK(cudaStreamSynchronize(h->stream));
+    h->nnzc = 0; h->nnza = 0; h->nnzb = 0;
+    *c_nnz = 0;
+    if (nprod_out) *nprod_out = 0;
+    h->state = 1;
+    return SPGEMM_OK;
+  }
+  ALLOC(h->nprod, sizeof(int64_t) * m);
+  ALLOC(h->grp1, m);
+  ALLOC(h->grp2, m);
+  ALLOC(h->perm1, sizeof(int32_t) * m);
+  ALLOC(h->perm2, sizeof(int32_t) * m);
+  ALLOC(h->tiles, scan_workspace_bytes(m));
+  if (h->timing) CK(cudaEventRecord(h->ev[0], h->stream));
+  if (h->validate) {
+    CK(launch_validate(h->stream, m, k, n, a_rpt, a_col, b_rpt, b_col, &dacc->err_flags));
+    ++launches;
+  }
+  // (1)+(2): n_prod per row (Alg. 2) and group ids / histogram
+  CK(launch_nprod_group(h->stream, m, a_rpt, a_col, b_rpt, static_cast<int64_t*>(h->nprod.p),
+                        static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h->sym_min_group), 3));
+  ++launches;
+  CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(h->hends + 0, a_rpt, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(h->hends + 1, a_rpt + m, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(h->hends + 2, b_rpt, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(h->hends + 3, b_rpt + k, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));  // sync 1: group sizes
+  h->snap1 = *h->hacc;
+  if (h->snap1.err_flags & 1) return fail(h, SPGEMM_ERR_INVALID_INPUT, "input validation failed (rpt not monotone or col out of range)");
+  h->nnza = h->hends[1] - h->hends[0];
+  h->nnzb = h->hends[3] - h->hends[2];
+  h->vw_log2 = auto_vw_log2(h);
+
+  const Offsets off1 = offsets_of(h->snap1.sym_rows, kNumSymGroups);
+  CK(launch_group_scatter(h->stream, m, static_cast<uint8_t*>(h->grp1.p), off1, dacc->cursor[0],
+                          static_cast<int32_t*>(h->perm1.p)));
+  ++launches;
+  if (h->timing) CK(cudaEventRecord(h->ev[1], h->stream));
+
+  // (3) symbolic hash counting per group
+  const long long n_opt = (long long)h->snap1.sym_rows[kSymOptimistic];
+  const long long n_glob = (long long)h->snap1.sym_rows[kSymGlobal];
+  if (n_opt > 0) ALLOC(h->overflow, sizeof(int32_t) * n_opt);
+  int glob_grid = 0;
+  long long slab_T = 0;
+  if (n_opt + n_glob > 0) {
+    const long long cap = std::min<long long>((long long)h->snap1.max_nprod, n);
+    slab_T = std::max<long long>(64, next_pow2(2 * std::max<long long>(cap, 1)));
+    const long long per = slab_T * 4;
+    const long long by_budget = std::max<long long>(1, h->ws_budget / per);
+    glob_grid = (int)std::min<long long>({n_opt + n_glob, 2LL * h->num_sms, by_budget});
+    ALLOC(h->slab_sym, (size_t)(glob_grid * per));
+  }
+  SymArgs sa{};
+  sa.a_rpt = a_rpt; sa.a_col = a_col; sa.b_rpt = b_rpt; sa.b_col = b_col;
+  sa.c_cnt = c_rpt + 1;
+  sa.vw_log2 = h->vw_log2;
+  sa.overflow_rows = static_cast<int32_t*>(h->overflow.p);
+  sa.overflow_count = &dacc->overflow_count;
+  const int T_opt = kSymGroups[kSymOptimistic].T, BS_opt = kSymGroups[kSymOptimistic].BS;
+  int lim = h->fill_limit > 0 ? h->fill_limit : T_opt / 2;
+  sa.fill_limit = std::max(1, std::min(lim, T_opt - BS_opt - 1));
+  sa.slab = static_cast<int*>(h->slab_sym.p);
+  sa.slab_T = slab_T;
+  sa.nprod = static_cast<int64_t*>(h->nprod.p);
+  sa.n = n;
+  const int32_t* perm1 = static_cast<const int32_t*>(h->perm1.p);
+  CK(fork(h));
+  for (int g = 0; g <= kSymOptimistic; ++g) {
+    const long long rows = (long long)h->snap1.sym_rows[g];
+    if (rows == 0) continue;
+    cudaStream_t s = group_stream(h, g);
+    if (h->timing) CK(cudaEventRecord(h->gstart[0][g], s));
+    SymArgs ga = sa;
+    ga.rows = perm1 + off1.off[g];
+    ga.nrows = rows;
+    CK(launch_symbolic_group(s, g, ga, h->num_sms));
+    ++launches;
+    if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
+      SymArgs gb = sa;
+      gb.rows = perm1 + off1.off[kSymGlobal];
+      gb.nrows = n_glob;
+      gb.dev_count = &dacc->overflow_count;
+      CK(launch_symbolic_global(s, gb, glob_grid));
+      ++launches;
+    }
+    if (h->timing) CK(cudaEventRecord(h->gstop[0][g], s));
+    h->gtimed[0][g] = true;
+  }
+  if (n_opt == 0 && n_glob > 0) {  // forced global group only
+    cudaStream_t s = group_stream(h, kSymGlobal);
+    if (h->timing) CK(cudaEventRecord(h->gstart[0][kSymGlobal], s));
+    SymArgs gb = sa;
+    gb.rows = perm1 + off1.off[kSymGlobal];
+    gb.nrows = n_glob;
+    gb.dev_count = nullptr;
+    CK(launch_symbolic_global(s, gb, glob_grid));
+    ++launches;
+    if (h->timing) CK(cudaEventRecord(h->gstop[0][kSymGlobal], s));
+    h->gtimed[0][kSymGlobal] = true;
+  }
+  CK(join(h));
+  if (h->timing) CK(cudaEventRecord(h->ev[2], h->stream));
+
+  // (4) rpt_C = prefix sum, fused with (6) grouping by nnz_i
+  int nl = 0;
+  CK(launch_scan_and_group(h->stream, m, c_rpt, static_cast<int64_t*>(h->nprod.p), a_rpt,
+                           static_cast<uint8_t*>(h->grp2.p), dacc, num_bounds(h->num_min_group),
+                           static_cast<long long*>(h->tiles.p), &nl));
+  launches += nl;
+  if (h->timing) CK(cudaEventRecord(h->ev[3], h->stream));
+  CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
+  buf_free(h, h->slab_sym);
+  buf_free(h, h->overflow);
+  CK(cudaStreamSynchronize(h->stream));  // sync 2: nnz(C) to the host
+  h->snap2 = *h->hacc;
+  h->nnzc = h->snap2.nnzc;
+  *c_nnz = h->nnzc;
+  if (nprod_out) *nprod_out = (int64_t)h->snap1.total_nprod;
+
+  spgemm_stats_t& st = h->stats;
+  st.nnz_a = h->nnza; st.nnz_b = h->nnzb; st.nnz_c = h->nnzc;
+  st.nprod = (int64_t)h->snap1.total_nprod;
+  st.max_row_nprod = (int64_t)h->snap1.max_nprod;
+  st.max_row_nnz = (int64_t)h->snap2.max_nnz;
+  for (int g = 0; g < kMaxGroups; ++g) {
+    st.sym_rows[g] = (int64_t)h->snap1.sym_rows[g];
+    st.sym_nprod[g] = (int64_t)h->snap1.sym_nprod[g];
+    st.sym_nnza[g] = (int64_t)h->snap1.sym_nnza[g];
+    st.num_rows[g] = (int64_t)h->snap2.num_rows[g];
+    st.num_nprod[g] = (int64_t)h->snap2.num_nprod[g];
+    st.num_nnza[g] = (int64_t)h->snap2.num_nnza[g];
+    st.num_nnzc[g] = (int64_t)h->snap2.num_nnzc[g];
+  }
+  st.sym_overflow_rows = h->snap2.overflow_count;
+  st.kernel_launches_symbolic = launches;
+  h->state = 1;
+  return SPGEMM_OK;
+}
+
+static spgemm_status_t ensure_perm2(spgemm_handle_t h) {
+  if (h->perm2_ready || h->m == 0) return SPGEMM_OK;
+  const Offsets off2 = offsets_of(h->snap2.num_rows, kNumNumGroups);
+  DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+  CK(launch_group_scatter(h->stream, h->m, static_cast<uint8_t*>(h->grp2.p), off2, dacc->cursor[1],
+                          static_cast<int32_t*>(h->perm2.p)));
+  h->stats.kernel_launches_numeric += 1;
+  h->perm2_ready = true;
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void* a_val, const void* b_val,
+                               int32_t* c_col, void* c_val) {
+  if (!h) return SPGEMM_ERR_INVALID_ARG;
+  if (h->state != 1) return fail(h, SPGEMM_ERR_BAD_STATE, "spgemm_numeric before spgemm_symbolic");
+  if (dt != SPGEMM_F32 && dt != SPGEMM_F64) return fail(h, SPGEMM_ERR_INVALID_ARG, "bad dtype");
+  if (h->nnzc > 0 && (!c_col || !c_val)) return fail(h, SPGEMM_ERR_INVALID_ARG, "NULL output pointer");
+  if (h->nnza > 0 && !a_val) return fail(h, SPGEMM_ERR_INVALID_ARG, "NULL a_val");
+  if (h->nnzb > 0 && !b_val) return fail(h, SPGEMM_ERR_INVALID_ARG, "NULL b_val");
+  DeviceGuard dg(h->device);
+  h->stats.kernel_launches_numeric = 0;
+  memset(h->gtimed[1], 0, sizeof h->gtimed[1]);
+  h->numeric_done = true;
+  if (h->timing) CK(cudaEventRecord(h->ev[4], h->stream));
+  if (h->m > 0 && h->nnzc > 0) {
+    spgemm_status_t s = ensure_perm2(h);
+    if (s != SPGEMM_OK) return s;
+    const bool fp64 = dt == SPGEMM_F64;
+    const long long vs = fp64 ? 8 : 4;
+    const Offsets off2 = offsets_of(h->snap2.num_rows, kNumNumGroups);
+    DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+    NumArgs na{};
+    na.a_rpt = h->a_rpt; na.a_col = h->a_col; na.a_val = a_val;
+    na.b_rpt = h->b_rpt; na.b_col = h->b_col; na.b_val = b_val;
+    na.c_rpt = h->c_rpt; na.c_col = c_col; na.c_val = c_val;
+    na.vw_log2 = h->vw_log2;
+    na.err_flags = &dacc->err_flags;
+    Buf slab;
+    const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
+    int glob_grid = 0;
+    if (n_glob > 0) {
+      const long long maxn = std::max<long long>(1, (long long)h->snap2.max_nnz);
+      const long long T = std::max<long long>(64, next_pow2(2 * maxn));
+      const long long stride = ((T * vs + T * 4 + (T / 4 + 1) * 4 + maxn * 4) + 255) & ~255LL;
+      const long long by_budget = std::max<long long>(1, h->ws_budget / stride);
+      glob_grid = (int)std::min<long long>({n_glob, 2LL * h->num_sms, by_budget});
+      s = buf_alloc(h, slab, (size_t)(glob_grid * stride));
+      if (s != SPGEMM_OK) return s;
+      na.slab = slab.p; na.slab_T = T; na.slab_stride = stride; na.max_nnz = maxn;
+    }
+    const int32_t* perm2 = static_cast<const int32_t*>(h->perm2.p);
+    CK(fork(h));
+    for (int g = 0; g < kNumNumGroups; ++g) {
+      const long long rows = (long long)h->snap2.num_rows[g];
+      if (rows == 0) continue;
+      cudaStream_t st = group_stream(h, g);
+      if (h->timing) CK(cudaEventRecord(h->gstart[1][g], st));
+      NumArgs ga = na;
+      ga.rows = perm2 + off2.off[g];
+      ga.nrows = rows;
+      if (g == kNumGlobal) CK(launch_numeric_global(st, fp64, ga, glob_grid));
+      else CK(launch_numeric_group(st, g, fp64, ga));
+      h->stats.kernel_launches_numeric += 1;
+      if (h->timing) CK(cudaEventRecord(h->gstop[1][g], st));
+      h->gtimed[1][g] = true;
+    }
+    CK(join(h));
+    buf_free(h, slab);
+  }
+  if (h->timing) CK(cudaEventRecord(h->ev[5], h->stream));
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t* out) {
+  if (!h || !out) return SPGEMM_ERR_INVALID_ARG;
+  DeviceGuard dg(h->device);
+  spgemm_stats_t st = h->stats;
+  if (h->state == 1 && h->m > 0 && h->timing) {
+    auto el = [&](cudaEvent_t a, cudaEvent_t b) -> float {
+      float ms = 0.f;
+      if (cudaEventSynchronize(b) != cudaSuccess || cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+        cudaGetLastError();
+        return -1.f;
+      }
+      return ms;
+    };
+    st.setup_ms = el(h->ev[0], h->ev[1]);
+    st.symbolic_ms = el(h->ev[1], h->ev[2]);
+    st.scan_ms = el(h->ev[2], h->ev[3]);
+    for (int g = 0; g < kMaxGroups; ++g) st.sym_group_ms[g] = h->gtimed[0][g] ? el(h->gstart[0][g], h->gstop[0][g]) : 0.f;
+    if (h->numeric_done) {
+      st.numeric_ms = el(h->ev[4], h->ev[5]);
+      for (int g = 0; g < kMaxGroups; ++g) st.num_group_ms[g] = h->gtimed[1][g] ? el(h->gstart[1][g], h->gstop[1][g]) : 0.f;
+      int flags = 0;
+      if (cudaMemcpy(&flags, &static_cast<DevAcc*>(h->acc.p)->err_flags, sizeof(int), cudaMemcpyDeviceToHost) == cudaSuccess &&
+          (flags & 2)) {
+        *out = st;
+        return fail(h, SPGEMM_ERR_INVALID_INPUT, "numeric row count disagreed with symbolic count");
+      }
+    }
+  }
+  st.workspace_bytes = h->ws_cur;
+  st.workspace_peak_bytes = h->ws_peak;
+  *out = st;
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_get_grouping(spgemm_handle_t h, int phase, int64_t* nprod, int32_t* perm, int64_t* offsets) {
+  if (!h || (phase != 1 && phase != 2)) return SPGEMM_ERR_INVALID_ARG;
+  if (h->state != 1) return fail(h, SPGEMM_ERR_BAD_STATE, "no symbolic result");
+  DeviceGuard dg(h->device);
+  if (h->m == 0) {
+    if (offsets) for (int g = 0; g <= (phase == 1 ? kNumSymGroups : kNumNumGroups); ++g) offsets[g] = 0;
+    return SPGEMM_OK;
+  }
+  if (phase == 2) {
+    spgemm_status_t s = ensure_perm2(h);
+    if (s != SPGEMM_OK) return s;
+  }
+  CK(cudaStreamSynchronize(h->stream));
+  if (nprod) CK(cudaMemcpy(nprod, h->nprod.p, sizeof(int64_t) * h->m, cudaMemcpyDeviceToHost));
+  if (perm) CK(cudaMemcpy(perm, phase == 1 ? h->perm1.p : h->perm2.p, sizeof(int32_t) * h->m, cudaMemcpyDeviceToHost));
+  if (offsets) {
+    const int ng = phase == 1 ? kNumSymGroups : kNumNumGroups;
+    const Offsets o = offsets_of(phase == 1 ? h->snap1.sym_rows : h->snap2.num_rows, ng);
+    for (int g = 0; g <= ng; ++g) offsets[g] = o.off[g];
+  }
+  return SPGEMM_OK;
+}
+
+spgemm_status_t spgemm_row_partition(spgemm_handle_t h, int64_t m, int64_t k, const int64_t* a_rpt,
+                                     const int32_t* a_col, const int64_t* b_rpt, int32_t nparts, int64_t* splits) {
+  if (!h || !splits || !a_rpt || !b_rpt || m < 0 || k < 0 || nparts < 1) return SPGEMM_ERR_INVALID_ARG;
+  if (!h->hacc) return fail(h, SPGEMM_ERR_BAD_STATE, "handle was not created successfully");
+  DeviceGuard dg(h->device);
+  Buf scan, tiles, dsplits;
+  spgemm_status_t s = buf_alloc(h, scan, sizeof(int64_t) * (m + 1));
+  if (s == SPGEMM_OK) s = buf_alloc(h, tiles, scan_workspace_bytes(m));
+  if (s == SPGEMM_OK) s = buf_alloc(h, dsplits, sizeof(int64_t) * (nparts + 1));
+  cudaError_t e = cudaSuccess;
+  if (s == SPGEMM_OK) {
+    int nl = 0;
+    e = launch_partition(h->stream, m, a_rpt, a_col, b_rpt, static_cast<int64_t*>(scan.p),
+                         static_cast<long long*>(tiles.p), nparts, static_cast<int64_t*>(dsplits.p), &nl);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(splits, dsplits.p, sizeof(int64_t) * (nparts + 1), cudaMemcpyDeviceToHost, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+  }
+  buf_free(h, scan);
+  buf_free(h, tiles);
+  buf_free(h, dsplits);
+  if (s != SPGEMM_OK) return s;
+  if (e != cudaSuccess) return fail_cuda(h, e, "spgemm_row_partition");
+  return SPGEMM_OK;
+}
+
+}  // extern "C"

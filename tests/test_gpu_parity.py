@@ -1,0 +1,296 @@
+"""Parity of the CUDA path (through the C ABI) with the CPU oracle (-m gpu).
+
+Comparison rule: rpt and col bit-exact; values within
+rtol * (|A||B|)_ij with rtol 1e-5 (fp32) / 1e-12 (fp64); integer-valued inputs bit-exact.
+Inputs are the seeded synthetic configs of BASELINE.json (synth/), same arrays on both sides.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from synth import Csr, from_coo
+
+pytestmark = pytest.mark.gpu
+
+RTOL = {np.float32: 1e-5, np.float64: 1e-12}
+
+
+@pytest.fixture(scope="module")
+def spg():
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    import paper_conf_icpp_nagasakanm17_b200 as P
+    P.load()
+    return P
+
+
+def _dev(spg, M: Csr, dtype):
+    return spg.CsrMatrix.from_host(M, "cuda", {np.float32: torch.float32, np.float64: torch.float64}[dtype])
+
+
+def run_gpu(spg, A: Csr, B: Csr, dtype, opts=None, handle=None):
+    own = handle is None
+    h = handle or spg.Handle()
+    try:
+        for k, v in (opts or {}).items():
+            h.set_option(k, v)
+        C = h.multiply(_dev(spg, A.astype(dtype), dtype), _dev(spg, B.astype(dtype), dtype))
+        torch.cuda.synchronize()
+        st = h.stats()
+        rpt, col, val = C.numpy()
+        return rpt, col, val, st, h.nprod
+    finally:
+        if own:
+            h.close()
+
+
+def assert_parity(got, ref, dtype, exact=False, what=""):
+    rpt, col, val = got[:3]
+    r_rpt, r_col, r_val, r_abs = ref
+    assert np.array_equal(rpt, r_rpt), f"{what}: rpt differs"
+    assert np.array_equal(col, r_col), f"{what}: col differs"
+    if exact:
+        assert np.array_equal(val, r_val), f"{what}: values not bit-exact"
+    else:
+        err = np.abs(val.astype(np.float64) - r_val.astype(np.float64))
+        bad = err > RTOL[dtype] * r_abs
+        assert not bad.any(), f"{what}: {bad.sum()} values out of tolerance, max err/S " \
+                              f"{(err / np.maximum(r_abs, 1e-300)).max():.3g}"
+
+
+def check(spg, A, B, dtype, exact=False, opts=None, what=""):
+    A = A.astype(dtype)
+    B = B.astype(dtype)
+    ref = oracle.spgemm(A, B, dtype)
+    got = run_gpu(spg, A, B, dtype, opts)
+    assert_parity(got, ref, dtype, exact, what)
+    _, total = oracle.nprod(A, B)
+    assert got[4] == total, f"{what}: nprod {got[4]} != {total}"
+    return got
+
+
+# ------------------------------------------------------------------ BASELINE configs
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_config1_poisson(spg, dtype):
+    A = synth.config("poisson64")
+    got = check(spg, A, A, dtype, exact=True, what="poisson64")
+    assert got[3]["nnz_c"] == 51972 and got[4] == 100104
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_config2_cant(spg, dtype):
+    A = synth.config("cant")
+    check(spg, A, A, dtype, what="cant")
+
+
+def test_config2_cant_int_exact(spg):
+    A = synth.config("cant", "int")
+    check(spg, A, A, np.float32, exact=True, what="cant int")
+
+
+def test_config3_webbase(spg):
+    A = synth.config("webbase")
+    got = check(spg, A, A, np.float32, what="webbase")
+    assert got[3]["sym_rows"][10] > 0  # heavy rows exercise the optimistic/global path
+
+
+def test_config3_webbase_int_exact(spg):
+    A = synth.config("webbase", "int")
+    check(spg, A, A, np.float32, exact=True, what="webbase int")
+
+
+@pytest.mark.parametrize("family", list(synth.MIXED))
+def test_config4_mixed(spg, family):
+    A = synth.config(f"mixed:{family}")
+    check(spg, A, A, np.float64, what=family)
+
+
+def test_rmat_s16(spg):
+    A = synth.rmat(16).with_values("uniform", 3)
+    check(spg, A, A, np.float32, what="rmat16")
+
+
+# ------------------------------------------------------------------ forced paths
+
+def _mixed_small():
+    A = synth.webbase_like(M=30000, seed=3, lmax=900, alpha=1.7)
+    return A.with_values("uniform", 4)
+
+
+@pytest.mark.parametrize("group", list(range(0, 12)))
+def test_forced_symbolic_group(spg, group):
+    A = _mixed_small()
+    ref = oracle.spgemm(A, A, np.float64)
+    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": group})
+    assert_parity(got, ref, np.float64, what=f"sym group>={group}")
+
+
+@pytest.mark.parametrize("group", list(range(0, 11)))
+def test_forced_numeric_group(spg, group):
+    A = _mixed_small()
+    ref = oracle.spgemm(A, A, np.float32)
+    got = run_gpu(spg, A, A, np.float32, {"num_min_group": group})
+    assert_parity(got, ref, np.float32, what=f"num group>={group}")
+
+
+def test_overflow_retry_in_global_memory(spg):
+    A = _mixed_small()
+    ref = oracle.spgemm(A, A, np.float64)
+    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16})
+    assert got[3]["sym_overflow_rows"] > 0
+    assert_parity(got, ref, np.float64, what="overflow")
+
+
+@pytest.mark.parametrize("lanes", [1, 2, 4, 8, 16, 32])
+def test_lanes_per_b_row(spg, lanes):
+    A = synth.MIXED["harbor"]().with_values("int", 1)
+    ref = oracle.spgemm(A, A, np.float64)
+    got = run_gpu(spg, A, A, np.float64, {"lanes": lanes})
+    assert_parity(got, ref, np.float64, exact=True, what=f"lanes={lanes}")
+
+
+def test_serial_streams(spg):
+    A = _mixed_small()
+    ref = oracle.spgemm(A, A, np.float64)
+    got = run_gpu(spg, A, A, np.float64, {"streams": 0})
+    assert_parity(got, ref, np.float64, what="no streams")
+
+
+# ------------------------------------------------------------------ edge cases
+
+def test_rectangular_and_identities(spg):
+    A = synth.random_sparse(700, 300, 0.02, seed=1).with_values("uniform", 1)
+    B = synth.random_sparse(300, 1100, 0.01, seed=2).with_values("uniform", 2)
+    check(spg, A, B, np.float64, what="rect")
+    idx = np.arange(300)
+    I = from_coo(300, 300, idx, idx, np.ones(300))
+    got = run_gpu(spg, A.astype(np.float32), I.astype(np.float32), np.float32)
+    assert np.array_equal(got[0], A.rpt) and np.array_equal(got[1], A.col)
+    assert np.array_equal(got[2], A.val.astype(np.float32))
+
+
+def test_structural_zero_and_degenerate(spg):
+    A = Csr(2, 2, np.array([0, 2, 4], np.int64), np.array([0, 1, 0, 1], np.int32),
+            np.array([1.0, 1.0, 1.0, -1.0]))
+    got = run_gpu(spg, A, A, np.float64)
+    assert got[0].tolist() == [0, 2, 4] and got[1].tolist() == [0, 1, 0, 1]
+    assert got[2].tolist() == [2.0, 0.0, 0.0, 2.0]
+    # m = 0
+    E = Csr(0, 5, np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0))
+    B = synth.random_sparse(5, 4, 0.5, seed=1).with_values()
+    got = run_gpu(spg, E, B, np.float64)
+    assert got[0].tolist() == [0] and len(got[1]) == 0
+    # A with no entries / empty rows
+    Z = Csr(3, 5, np.zeros(4, np.int64), np.zeros(0, np.int32), np.zeros(0))
+    got = run_gpu(spg, Z, B, np.float32)
+    assert got[0].tolist() == [0, 0, 0, 0]
+    # empty rows interleaved
+    A2 = synth.random_sparse(500, 500, 0.003, seed=9).with_values("int", 2)
+    assert (np.diff(A2.rpt) == 0).any()
+    check(spg, A2, A2, np.float64, exact=True, what="sparse empty rows")
+
+
+def test_duplicates_unsorted(spg):
+    A = synth.random_sparse(400, 300, 0.05, seed=31, dup=True).with_values("int", 4)
+    B = synth.random_sparse(300, 350, 0.05, seed=32, unsorted=True).with_values("int", 5)
+    check(spg, A, B, np.float64, exact=True, what="dup/unsorted")
+
+
+def test_large_column_indices(spg):
+    n = 2**31 - 2
+    rng = np.random.default_rng(0)
+    B = from_coo(64, n, rng.integers(0, 64, 500), rng.integers(0, n, 500), rng.uniform(-1, 1, 500))
+    A = synth.random_sparse(50, 64, 0.2, seed=4).with_values("uniform", 5)
+    check(spg, A, B, np.float64, what="huge n")
+
+
+def test_row_slice_offset_pointer(spg):
+    A = synth.MIXED["accelerator"]().with_values("uniform", 2)
+    ref = oracle.spgemm(A, A, np.float64)
+    r0, r1 = 1000, 50000
+    dA = _dev(spg, A, np.float64)
+    sl = spg.CsrMatrix(r1 - r0, A.n, dA.rpt[r0:r1 + 1].contiguous(), dA.col, dA.val)  # a_rpt[0] != 0
+    with spg.Handle() as h:
+        C = h.multiply(sl, dA)
+        rpt, col, val = C.numpy()
+    s, e = ref[0][r0], ref[0][r1]
+    assert np.array_equal(rpt, ref[0][r0:r1 + 1] - s)
+    assert np.array_equal(col, ref[1][s:e])
+    assert np.all(np.abs(val - ref[2][s:e]) <= 1e-12 * ref[3][s:e])
+
+
+def test_structure_reuse_and_torch_allocator(spg):
+    A = synth.MIXED["ship"]()
+    A1 = A.with_values("int", 1)
+    A2 = A.with_values("int", 2)
+    r1 = oracle.spgemm(A1, A1, np.float64)
+    r2 = oracle.spgemm(A2, A2, np.float64)
+    with spg.Handle(torch_allocator=True) as h:
+        d1 = _dev(spg, A1, np.float64)
+        C = h.multiply(d1, d1)
+        assert_parity(C.numpy() + (None,), r1, np.float64, exact=True, what="first")
+        d2 = _dev(spg, A2, np.float64)
+        h.numeric(d2.val, d2.val, C.col, C.val)   # same structure, new values
+        assert_parity(C.numpy() + (None,), r2, np.float64, exact=True, what="reuse")
+        st = h.stats()
+        assert st["workspace_peak_bytes"] > 0
+
+
+# ------------------------------------------------------------------ intermediate steps
+
+def test_nprod_and_grouping(spg):
+    A = _mixed_small()
+    nprod_ref, total = oracle.nprod(A, A)
+    ref_rpt = oracle.symbolic(A, A)
+    with spg.Handle() as h:
+        dA = _dev(spg, A, np.float32)
+        h.symbolic(dA, dA)
+        nprod, perm, off = h.grouping(1)
+        nprod2, perm2, off2 = h.grouping(2)
+    assert np.array_equal(nprod, nprod_ref) and h.nprod == total
+    for ph, (p, o, keys) in ((1, (perm, off, nprod_ref)), (2, (perm2, off2, np.diff(ref_rpt)))):
+        upper = spg.group_bounds(ph)
+        want = oracle.bin_of(keys, upper)
+        nonempty = np.flatnonzero(want >= 0)
+        assert o[-1] == len(nonempty)
+        assert np.array_equal(np.sort(p[:o[-1]]), nonempty)       # a permutation of grouped rows
+        for g in range(len(o) - 1):
+            rows = p[o[g]:o[g + 1]]
+            assert np.all(want[rows] == g), f"phase {ph} group {g}"
+
+
+def test_row_partition(spg):
+    A = synth.config("webbase")
+    nprod_ref, total = oracle.nprod(A, A)
+    excl = np.concatenate([[0], np.cumsum(nprod_ref)])
+    with spg.Handle() as h:
+        dA = _dev(spg, A, np.float32)
+        for P in (1, 2, 3, 8):
+            s = h.row_partition(dA, dA, P)
+            want = [int(np.searchsorted(excl, (total * p) // P, side="left")) for p in range(P)] + [A.m]
+            assert s.tolist() == want
+
+
+# ------------------------------------------------------------------ full size, sampled
+
+@pytest.mark.slow
+def test_rmat_s20_sampled(spg):
+    A = synth.rmat(20).with_values("uniform", 7)
+    with spg.Handle() as h:
+        dA = _dev(spg, A, np.float32)
+        C = h.multiply(dA, dA)
+        rpt, col, val = C.numpy()
+    A32 = A.astype(np.float32)
+    assert rpt[0] == 0 and np.all(np.diff(rpt) >= 0)
+    rng = np.random.default_rng(0)
+    heavy = np.argsort(np.diff(rpt))[-20:]
+    for r in np.concatenate([rng.integers(0, A.m, 200), heavy]):
+        S = oracle.row_slice(A32, int(r), int(r) + 1)
+        r_rpt, r_col, r_val, r_abs = oracle.spgemm(S, A32, np.float32)
+        s, e = rpt[r], rpt[r + 1]
+        assert e - s == r_rpt[1]
+        assert np.array_equal(col[s:e], r_col)
+        assert np.all(np.abs(val[s:e] - r_val) <= 1e-5 * r_abs)
