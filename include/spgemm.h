@@ -122,7 +122,9 @@ typedef enum {
     SPGEMM_OPT_VALIDATE = 4,        /* 1 = O(nnz) input validation in spgemm_symbolic */
     SPGEMM_OPT_LANES = 5,           /* lanes per B row (power of two 1..32), 0 = auto */
     SPGEMM_OPT_WORKSPACE_BUDGET = 6,/* max bytes for global-memory hash tables */
-    SPGEMM_OPT_TIMING = 7           /* 1 = per-group CUDA-event timing (default 1) */
+    SPGEMM_OPT_TIMING = 7,          /* 1 = per-group CUDA-event timing (default 1) */
+    SPGEMM_OPT_LONG_ROW = 8         /* CTA-per-row groups: B rows longer than v are walked by
+                                       the whole CTA (0 = auto, -1 = off) */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

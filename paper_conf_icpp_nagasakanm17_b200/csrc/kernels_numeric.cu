@@ -8,11 +8,14 @@
 // above the largest shared-memory group use a per-CTA global-memory slab.
 //
 // B200 deviation in (b)/(c): the paper's rank sort compares every entry with
-// every other (O(nnz_i^2) per row).  Here the gather scatters entries into NB = T/4 buckets
-// of the row's column range [lo, hi] (lo/hi tracked with shared atomics at insertion), and
-// each entry's rank = start of its bucket + number of smaller keys in the same bucket — the
-// paper's comparison rank restricted to the bucket.  Keys are distinct, so the output is
-// identical to any correct sort.
+// every other (O(nnz_i^2) per row).  Here, with [lo, hi] the row's column range (a group
+// min/max over the table after accumulation):
+//   (c1) range/NB <= 4 (banded/FEM rows): entries are scattered into NB buckets of width
+//        <= 4 and rank = bucket start + #smaller keys in the bucket (the paper's comparison
+//        rank restricted to a bucket) — a prefix count when the range fits NB;
+//   (c2) wider ranges in shared memory: bitonic sort of the compacted slot indices;
+//   (c3) global-memory rows: bitmap over [lo, hi] + prefix popcounts.
+// Keys are distinct, so every path writes the identical, sorted row.
 #include <climits>
 
 #include "spgemm_internal.cuh"
@@ -21,90 +24,207 @@ namespace spg {
 
 namespace {
 
-template <typename VT>
-__device__ __forceinline__ void add_value(VT* p, VT v) { atomicAdd(p, v); }
+struct NoStop {
+  __device__ __forceinline__ bool operator()() const { return false; }
+};
 
-template <typename VT, int TPR, typename SIdx>
-__device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, int* K, VT* V, int* Bc,
-                                        SIdx* S, unsigned mask, int NB, int* lohi, long long* ws) {
+template <typename VT>
+struct Vec16;  // 16-byte vector of VT
+template <>
+struct Vec16<float> { using T = float4; static __device__ __forceinline__ float4 zero() { return make_float4(0.f, 0.f, 0.f, 0.f); } };
+template <>
+struct Vec16<double> { using T = double2; static __device__ __forceinline__ double2 zero() { return make_double2(0.0, 0.0); } };
+
+// One row: (0) init, (a) accumulate, (b) gather into buckets, (c) rank + write.
+// Kp/Vp: the key/value tables (shared or global); Keys/Vals: their probe/add accessors.
+template <typename VT, int TPR, bool GLOBAL, typename Keys, typename Vals, typename SIdx>
+__device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, const Keys& K, const Vals& V,
+                                        int* Kp, VT* Vp, int* Bc, SIdx* S, unsigned mask, int NB, int* lohi,
+                                        long long* ws, int* s_list, int* s_lcnt) {
   const int t = Grp<TPR>::lane();
   const unsigned T = mask + 1;
-  // (0) init: keys <- -1 (Alg. 5 precondition), values <- 0
-  for (unsigned s = t; s < T; s += TPR) { K[s] = -1; V[s] = VT(0); }
-  if (t == 0) { lohi[0] = INT_MAX; lohi[1] = -1; }
+  // (0) keys <- -1 (Alg. 5 precondition), values <- 0; 16-byte stores
+  {
+    int4* k4 = reinterpret_cast<int4*>(Kp);
+    for (unsigned s = t; s < T / 4; s += TPR) k4[s] = make_int4(-1, -1, -1, -1);
+    using V16 = typename Vec16<VT>::T;
+    V16* v16 = reinterpret_cast<V16*>(Vp);
+    constexpr unsigned per = 16 / sizeof(VT);
+    for (unsigned s = t; s < T / per; s += TPR) v16[s] = Vec16<VT>::zero();
+  }
   Grp<TPR>::sync();
 
   // (a) accumulate
-  if (active) {
-    const VT* __restrict__ av = static_cast<const VT*>(a.a_val);
-    const VT* __restrict__ bv = static_cast<const VT*>(a.b_val);
-    const long long a0 = a.a_rpt[row], a1 = a.a_rpt[row + 1];
-    const int vwl = a.vw_log2;
-    const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = TPR >> vwl;
-    for (long long j = a0 + sub; j < a1; j += nsub) {
-      const int kk = __ldg(a.a_col + j);
-      const VT aik = av[j];
-      const long long b0 = __ldg(a.b_rpt + kk), b1 = __ldg(a.b_rpt + kk + 1);
-      for (long long q = b0 + lane; q < b1; q += vw) {
-        const int key = __ldg(a.b_col + q);
-        const VT prod = aik * bv[q];  // value <- a_ik b_kj (Alg. 1)
-        bool ins;
-        const unsigned s = hash_slot(K, mask, key, ins);
-        if (ins) { atomicMin(&lohi[0], key); atomicMax(&lohi[1], key); }
-        add_value(V + s, prod);
-      }
+  {
+    auto f = [&](int key, VT prod) {  // prod = a_ik * b_kj (Alg. 1 "value")
+      bool ins;
+      const unsigned s = probe(K, mask, key, ins);
+      V.add(s, prod);
+    };
+    const int long_len = TPR > 32 ? a.long_len : 0;
+    if (active)
+      for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
+                                        static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
+                                        long_len);
+    if constexpr (TPR > 32) {
+      if (long_len > 0)
+        for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
+                                           static_cast<const VT*>(a.b_val), active, row, t, TPR, long_len, s_list,
+                                           s_lcnt, f, NoStop{});
     }
   }
   Grp<TPR>::sync();
 
-  // (b) gather: bucket histogram over the column range
-  const int lo = lohi[0], hi = lohi[1];
-  int shift = 0, nb = 0;
-  if (hi >= lo) {
-    const unsigned R = (unsigned)(hi - lo);
-    while ((R >> shift) >= (unsigned)NB) ++shift;
-    nb = (int)(R >> shift) + 1;
-  }
-  for (int b = t; b <= nb; b += TPR) Bc[b] = 0;
-  Grp<TPR>::sync();
-  for (unsigned s = t; s < T; s += TPR) {
-    const int key = K[s];
-    if (key >= 0) atomicAdd(&Bc[1 + ((key - lo) >> shift)], 1);
-  }
-  Grp<TPR>::sync();
-  long long n_total;
+  // (b) gather: column range [lo, hi] of the row (group min/max over the table)
+  const int4* k4 = reinterpret_cast<const int4*>(Kp);
   {
-    const int per = (nb + TPR - 1) / TPR;
-    const int b0 = 1 + t * per;
-    const int b1 = min(nb + 1, b0 + per);
-    long long loc = 0;
-    for (int b = b0; b < b1; ++b) loc += Bc[b];
-    long long run = Grp<TPR>::excl_scan(loc, &n_total, ws);
-    for (int b = b0; b < b1; ++b) { const int c = Bc[b]; Bc[b] = (int)run; run += c; }
+    int mn = INT_MAX, mx = -1;
+    for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+      const int4 kv = k4[s4];
+      mx = max(max(mx, kv.x), max(kv.y, max(kv.z, kv.w)));
+      mn = min(mn, kv.x < 0 ? INT_MAX : kv.x);
+      mn = min(mn, kv.y < 0 ? INT_MAX : kv.y);
+      mn = min(mn, kv.z < 0 ? INT_MAX : kv.z);
+      mn = min(mn, kv.w < 0 ? INT_MAX : kv.w);
+    }
+    Grp<TPR>::minmax(mn, mx, lohi);
   }
-  Grp<TPR>::sync();
-  for (unsigned s = t; s < T; s += TPR) {
-    const int key = K[s];
-    if (key >= 0) S[atomicAdd(&Bc[1 + ((key - lo) >> shift)], 1)] = (SIdx)s;
-  }
-  Grp<TPR>::sync();
-
-  // (c) rank = bucket start + #smaller keys in the bucket; write C
-  if (active) {
-    const long long c0 = a.c_rpt[row];
-    const long long cn = a.c_rpt[row + 1] - c0;
-    if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
-    VT* __restrict__ cv = static_cast<VT*>(a.c_val);
-    for (long long p = t; p < n_total; p += TPR) {
-      const unsigned s = S[p];
-      const int key = K[s];
-      const int b = (key - lo) >> shift;
-      const int st = Bc[b], en = Bc[b + 1];
-      int r = st;
-      for (int q = st; q < en; ++q) r += (K[S[q]] < key);
-      if (r < cn) {
-        a.c_col[c0 + r] = key;
-        cv[c0 + r] = V[s];
+  const int lo = lohi[0], hi = lohi[1];
+  const long long c0 = active ? a.c_rpt[row] : 0;
+  const long long cn = active ? a.c_rpt[row + 1] - c0 : 0;
+  VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+  int32_t* __restrict__ cc = a.c_col + c0;
+  long long n_total = 0;
+  if constexpr (GLOBAL) {
+    // (c) global-memory rows: bitmap rank over [lo, hi]; rank(key) = #set bits below it
+    // (prefix popcount per 32-bit word + popc of the partial word).  Bc = bitmap, S = prefix.
+    const int W = hi >= lo ? (int)(((unsigned)(hi - lo)) >> 5) + 1 : 0;
+    unsigned* bits = reinterpret_cast<unsigned*>(Bc);
+    for (int w = t; w < W; w += TPR) bits[w] = 0u;
+    Grp<TPR>::sync();
+    for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+      const int4 kv = k4[s4];
+      if (kv.x >= 0) atomicOr(bits + ((kv.x - lo) >> 5), 1u << ((kv.x - lo) & 31));
+      if (kv.y >= 0) atomicOr(bits + ((kv.y - lo) >> 5), 1u << ((kv.y - lo) & 31));
+      if (kv.z >= 0) atomicOr(bits + ((kv.z - lo) >> 5), 1u << ((kv.z - lo) & 31));
+      if (kv.w >= 0) atomicOr(bits + ((kv.w - lo) >> 5), 1u << ((kv.w - lo) & 31));
+    }
+    Grp<TPR>::sync();
+    {
+      const int per = (W + TPR - 1) / TPR;
+      const int w0 = t * per, w1 = min(W, w0 + per);
+      long long loc = 0;
+      for (int w = w0; w < w1; ++w) loc += __popc(bits[w]);
+      long long run = Grp<TPR>::excl_scan(loc, &n_total, ws);
+      for (int w = w0; w < w1; ++w) { S[w] = (SIdx)run; run += __popc(bits[w]); }
+    }
+    Grp<TPR>::sync();
+    if (active) {
+      if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
+      for (unsigned s = t; s < T; s += TPR) {
+        const int key = Kp[s];
+        if (key < 0) continue;
+        const unsigned d = (unsigned)(key - lo);
+        const int r = (int)S[d >> 5] + __popc(bits[d >> 5] & ((1u << (d & 31)) - 1u));
+        if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
+      }
+    }
+  } else {
+    int shift = 0, nb = 0;
+    if (hi >= lo) {
+      const unsigned R = (unsigned)(hi - lo);
+      while ((R >> shift) >= (unsigned)NB) ++shift;
+      nb = (int)(R >> shift) + 1;
+    }
+    if (shift <= 2) {
+      // (c1) bucket rank: NB buckets of width 2^shift <= 4 over [lo, hi]; rank = bucket start
+      // + #smaller keys in the same bucket (the paper's comparison rank, within a bucket).
+      for (int b = t; b <= nb; b += TPR) Bc[b] = 0;
+      Grp<TPR>::sync();
+      for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+        const int4 kv = k4[s4];
+        if (kv.x >= 0) atomicAdd(&Bc[1 + ((kv.x - lo) >> shift)], 1);
+        if (kv.y >= 0) atomicAdd(&Bc[1 + ((kv.y - lo) >> shift)], 1);
+        if (kv.z >= 0) atomicAdd(&Bc[1 + ((kv.z - lo) >> shift)], 1);
+        if (kv.w >= 0) atomicAdd(&Bc[1 + ((kv.w - lo) >> shift)], 1);
+      }
+      Grp<TPR>::sync();
+      {
+        const int per = (nb + TPR - 1) / TPR;
+        const int b0 = 1 + t * per;
+        const int b1 = min(nb + 1, b0 + per);
+        long long loc = 0;
+        for (int b = b0; b < b1; ++b) loc += Bc[b];
+        long long run = Grp<TPR>::excl_scan(loc, &n_total, ws);
+        for (int b = b0; b < b1; ++b) { const int c = Bc[b]; Bc[b] = (int)run; run += c; }
+      }
+      Grp<TPR>::sync();
+      for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+        const int4 kv = k4[s4];
+        const unsigned s = 4 * s4;
+        if (kv.x >= 0) S[atomicAdd(&Bc[1 + ((kv.x - lo) >> shift)], 1)] = (SIdx)(s);
+        if (kv.y >= 0) S[atomicAdd(&Bc[1 + ((kv.y - lo) >> shift)], 1)] = (SIdx)(s + 1);
+        if (kv.z >= 0) S[atomicAdd(&Bc[1 + ((kv.z - lo) >> shift)], 1)] = (SIdx)(s + 2);
+        if (kv.w >= 0) S[atomicAdd(&Bc[1 + ((kv.w - lo) >> shift)], 1)] = (SIdx)(s + 3);
+      }
+      Grp<TPR>::sync();
+      if (active) {
+        if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
+        for (int p = t; p < (int)n_total; p += TPR) {
+          const unsigned s = S[p];
+          const int key = Kp[s];
+          const int b = (key - lo) >> shift;
+          const int st = Bc[b], en = Bc[b + 1];
+          int r = st;
+          for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
+          if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
+        }
+      }
+    } else {
+      // (c2) wide, clustered ranges: compact the slot indices, bitonic-sort them by key in
+      // shared memory (n' = next_pow2(n) <= the group's nnz bound), write C coalesced.
+      int* cnt = Bc;
+      if (t == 0) *cnt = 0;
+      Grp<TPR>::sync();
+      for (unsigned s = t; s < T; s += TPR) {
+        const bool occ = Kp[s] >= 0;
+        const unsigned bal = __ballot_sync(Grp<TPR>::mask(), occ);
+        if (bal) {  // uniform across the row group
+          const int lead = __ffs(bal) - 1;
+          int base = 0;
+          if ((threadIdx.x & 31) == lead) base = atomicAdd(cnt, __popc(bal));
+          base = __shfl_sync(Grp<TPR>::mask(), base, lead);
+          if (occ) S[base + __popc(bal & ((1u << (threadIdx.x & 31)) - 1u))] = (SIdx)s;
+        }
+      }
+      Grp<TPR>::sync();
+      const int n = *cnt;
+      n_total = n;
+      int np2 = 1;
+      while (np2 < n) np2 <<= 1;
+      constexpr SIdx kSent = (SIdx)~SIdx(0);
+      for (int p = n + t; p < np2; p += TPR) S[p] = kSent;
+      Grp<TPR>::sync();
+      auto keyof = [&](SIdx x) { return x == kSent ? INT_MAX : Kp[x]; };
+      for (int k = 2; k <= np2; k <<= 1) {
+        for (int j = k >> 1; j > 0; j >>= 1) {
+          for (int q = t; q < (np2 >> 1); q += TPR) {
+            const int i = ((q & ~(j - 1)) << 1) | (q & (j - 1));
+            const int l = i | j;
+            const SIdx x = S[i], y = S[l];
+            const bool up = (i & k) == 0;
+            if ((keyof(x) > keyof(y)) == up) { S[i] = y; S[l] = x; }
+          }
+          Grp<TPR>::sync();
+        }
+      }
+      if (active) {
+        if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
+        for (int p = t; p < n && p < cn; p += TPR) {
+          const unsigned s = S[p];
+          cc[p] = Kp[s];
+          cv[p] = Vp[s];
+        }
       }
     }
   }
@@ -117,36 +237,40 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   __shared__ long long ws[33];
   constexpr int RPB = BS / TPR;
   __shared__ int s_lohi[2 * RPB];
+  __shared__ int s_list[TPR > 32 ? kLongChunk : 1], s_lcnt;
   constexpr int NB = num_nbuckets(T);
   constexpr int RB = num_row_bytes<VT>(T, UPPER);
   const int g = threadIdx.x / TPR;
   unsigned char* base = smem_raw + g * RB;
-  VT* V = reinterpret_cast<VT*>(base);
-  int* K = reinterpret_cast<int*>(base + T * sizeof(VT));
-  int* Bc = K + T;
+  VT* Vp = reinterpret_cast<VT*>(base);
+  int* Kp = reinterpret_cast<int*>(base + T * sizeof(VT));
+  int* Bc = Kp + T;
   uint16_t* S = reinterpret_cast<uint16_t*>(Bc + NB + 1);
   const long long ridx = (long long)blockIdx.x * RPB + g;
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : 0;
-  num_row<VT, TPR, uint16_t>(a, active, row, K, V, Bc, S, T - 1, NB, s_lohi + 2 * g, ws);
+  num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
+                   s_lohi + 2 * g, ws, s_list, &s_lcnt);
 }
 
 template <typename VT>
 __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_lohi[2];
+  __shared__ int s_list[kLongChunk], s_lcnt;
   unsigned char* slab = static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride;
-  VT* V = reinterpret_cast<VT*>(slab);
-  int* K = reinterpret_cast<int*>(V + a.slab_T);
-  int* Bc = K + a.slab_T;
-  int* S = Bc + a.slab_T / 4 + 1;
+  VT* Vp = reinterpret_cast<VT*>(slab);
+  int* Kp = reinterpret_cast<int*>(Vp + a.slab_T);
+  int* Bc = Kp + a.slab_T;              // bitmap over [lo, hi]: bitmap_words ints
+  int* S = Bc + a.bitmap_words;         // prefix popcount per bitmap word
   for (long long i = blockIdx.x; i < a.nrows; i += gridDim.x) {
     const int row = a.rows[i];
     const long long n = a.c_rpt[row + 1] - a.c_rpt[row];
     long long T = 64;
     while (T < 2 * n) T <<= 1;
     if (T > a.slab_T) T = a.slab_T;
-    num_row<VT, 1024, int>(a, true, row, K, V, Bc, S, (unsigned)(T - 1), (int)(T / 4), s_lohi, ws);
+    num_row<VT, 1024, true>(a, true, row, GKeys{Kp}, GVals<VT>{Vp}, Kp, Vp, Bc, S, (unsigned)(T - 1), 0,
+                      s_lohi, ws, s_list, &s_lcnt);
   }
 }
 
@@ -154,7 +278,7 @@ template <typename VT, int T, int TPR, int BS, long long UPPER>
 cudaError_t launch_num(cudaStream_t s, const NumArgs& a) {
   constexpr int RPB = BS / TPR;
   constexpr int smem = RPB * num_row_bytes<VT>(T, UPPER);
-  static_assert(smem + 33 * 8 + 8 * RPB <= kSmemLimit, "numeric table too large");
+  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 <= kSmemLimit, "numeric table too large");
   static bool configured = false;
   if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(k_num_smem<VT, T, TPR, BS, UPPER>,

@@ -50,20 +50,21 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
   }
 #pragma unroll
   for (int off = LPR / 2; off > 0; off >>= 1) np += __shfl_xor_sync(0xffffffffu, np, off);
-  if (row < m && l == 0) {
+  int g = 0xFF;
+  const bool lead = row < m && l == 0;
+  if (lead) {
     nprod[row] = np;
-    int g = 0xFF;
-    if (np == 0) {
-      c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
-    } else {
-      g = group_of(np, bd);
-      atomicAdd(&s_rows[g], 1ull);
-      atomicAdd(&s_np[g], (unsigned long long)np);
-      atomicAdd(&s_nza[g], (unsigned long long)(a1 - a0));
-    }
+    if (np == 0) c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
+    else g = group_of(np, bd);
     grp[row] = (uint8_t)g;
-    atomicAdd(&s_total, (unsigned long long)np);
-    atomicMax(&s_max, (unsigned long long)np);
+  }
+  {
+    const unsigned long long v[3] = {1ull, (unsigned long long)np, (unsigned long long)(a1 - a0)};
+    unsigned long long* const d[3] = {s_rows, s_np, s_nza};
+    warp_group_add<3>(lead && g != 0xFF, g, v, d);
+    const unsigned long long tot = warp_sum_u64(lead ? (unsigned long long)np : 0ull);
+    const unsigned long long mx = warp_max_u64(lead ? (unsigned long long)np : 0ull);
+    if ((threadIdx.x & 31) == 0) { atomicAdd(&s_total, tot); atomicMax(&s_max, mx); }
   }
   __syncthreads();
   if (threadIdx.x < kMaxGroups && s_rows[threadIdx.x]) {
@@ -139,21 +140,22 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(
 #pragma unroll
   for (int e = 0; e < kScanItems; ++e) {
     const long long i = base + e * kSetupThreads + threadIdx.x;
-    if (i < m) {
-      const long long v = x[i];
-      s += v;
-      if (grouping) {
-        int g = 0xFF;
-        if (v > 0) {
-          g = group_of(v, bd);
-          atomicAdd(&s_rows[g], 1ull);
-          atomicAdd(&s_nzc[g], (unsigned long long)v);
-          atomicAdd(&s_np[g], (unsigned long long)nprod[i]);
-          atomicAdd(&s_nza[g], (unsigned long long)(a_rpt[i + 1] - a_rpt[i]));
-          atomicMax(&s_max, (unsigned long long)v);
-        }
+    const long long v = i < m ? x[i] : 0;
+    s += v;
+    if (grouping) {  // block-uniform branch
+      int g = 0xFF;
+      if (i < m) {
+        if (v > 0) g = group_of(v, bd);
         grp2[i] = (uint8_t)g;
       }
+      const bool valid = g != 0xFF;
+      const unsigned long long vv[4] = {1ull, (unsigned long long)v,
+                                        valid ? (unsigned long long)nprod[i] : 0ull,
+                                        valid ? (unsigned long long)(a_rpt[i + 1] - a_rpt[i]) : 0ull};
+      unsigned long long* const d[4] = {s_rows, s_nzc, s_np, s_nza};
+      warp_group_add<4>(valid, g, vv, d);
+      const unsigned long long mx = warp_max_u64(valid ? (unsigned long long)v : 0ull);
+      if ((threadIdx.x & 31) == 0 && mx) atomicMax(&s_max, mx);
     }
   }
   const long long tot = block_sum_ll(s, ws);

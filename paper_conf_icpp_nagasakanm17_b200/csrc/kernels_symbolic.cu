@@ -2,28 +2,33 @@
 // hash tables (§III-B), one kernel per group (Table I, B200 values in
 // spgemm_internal.cuh).
 //
-// Thread assignment (Alg. 3/4) generalised: a row is owned by TPR threads
-// (4..32 lanes = PWARP/ROW family, or a whole CTA = TB/ROW); inside the row, sub-groups of
-// VW = 2^vw_log2 lanes take successive non-zeros of A (Alg. 4's "one warp per a_ik") and
-// stride VW over the B row (Alg. 4's "one thread per b_kj").  VW is chosen from the mean B
-// row length so short B rows (graphs) do not idle 32-lane warps; VW = 1 is exactly Alg. 3.
+// Thread assignment (Alg. 3/4) generalised in for_each_product: a row is
+// owned by TPR threads (4..32 lanes = the PWARP/ROW family, or a whole CTA = TB/ROW); inside
+// the row, sub-groups of VW lanes take successive non-zeros of A (Alg. 4 "one warp for each
+// non-zero element of matrix A") and stride VW over the B row (Alg. 4 "one thread for each
+// non-zero element of matrix B").  VW = 1 is exactly Alg. 3.
 //
-// Hash table: Alg. 5 in shared memory (hash_insert), t_size a power of two >= 2x the
-// group's n_prod bound, so it cannot overflow.  The optimistic group (rows above the last
-// bound) uses the largest table and aborts a row once it has found `fill_limit` distinct
-// keys; the row index is recorded and the row is recounted in a global-memory table sized
-// from its n_prod by k_sym_global.
+// Hash table: Alg. 5 in shared memory, t_size a power of two >= 2x the group's n_prod bound,
+// so it cannot overflow.  The optimistic group (rows above the last bound) uses the largest
+// table and aborts a row once it has found `fill_limit` distinct keys; the row index is
+// recorded and the row is recounted in a global-memory table sized from its n_prod
+// by k_sym_global.
 #include "spgemm_internal.cuh"
 
 namespace spg {
 
 namespace {
 
+struct NoStop {
+  __device__ __forceinline__ bool operator()() const { return false; }
+};
+
 template <int T, int TPR, int BS, bool OPT>
 __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   extern __shared__ __align__(16) int smem[];
   __shared__ long long ws[33];
-  __shared__ int s_cnt, s_abort;
+  __shared__ int s_cnt, s_abort, s_lcnt;
+  __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
   constexpr int RPB = BS / TPR;
   static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
   const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
@@ -31,29 +36,43 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   const long long ridx = (long long)blockIdx.x * RPB + g;
 
   int4* t4 = reinterpret_cast<int4*>(table);
+#pragma unroll 4
   for (int s = t; s < T / 4; s += TPR) t4[s] = make_int4(-1, -1, -1, -1);
   if (OPT && threadIdx.x == 0) { s_cnt = 0; s_abort = 0; }
   Grp<TPR>::sync();
 
-  int cnt = 0, row = -1;
-  if (ridx < a.nrows) {
-    row = a.rows[ridx];
-    const long long a0 = a.a_rpt[row], a1 = a.a_rpt[row + 1];
-    const int vwl = a.vw_log2;
-    const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = TPR >> vwl;
-    for (long long j = a0 + sub; j < a1; j += nsub) {
-      if (OPT && ld_volatile(&s_abort)) break;
-      const int kk = __ldg(a.a_col + j);
-      const long long b0 = __ldg(a.b_rpt + kk), b1 = __ldg(a.b_rpt + kk + 1);
-      for (long long q = b0 + lane; q < b1; q += vw) {
-        const int key = __ldg(a.b_col + q);
-        if constexpr (OPT) {
-          if (ld_volatile(&s_abort)) break;
-          if (hash_insert(table, T - 1, key) && atomicAdd(&s_cnt, 1) + 1 >= a.fill_limit) s_abort = 1;
-        } else {
-          cnt += hash_insert(table, T - 1, key);
-        }
-      }
+  int cnt = 0;
+  const bool active = ridx < a.nrows;
+  const int row = active ? a.rows[ridx] : -1;
+  const SKeys K{smem_u32(table)};
+  const int long_len = TPR > 32 ? a.long_len : 0;
+  if constexpr (OPT) {
+    const unsigned ab = smem_u32(&s_abort);
+    auto stop = [ab]() { return lds_s32(ab) != 0; };
+    auto f = [&](int key, int) {
+      bool ins;
+      probe(K, T - 1, key, ins);
+      if (ins && atomicAdd(&s_cnt, 1) + 1 >= a.fill_limit) s_abort = 1;
+    };
+    if (active)
+      for_each_product<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
+                                         a.vw_log2, f, stop, long_len);
+    if (long_len > 0)
+      for_long_products<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
+                                          TPR, long_len, s_list, &s_lcnt, f, stop);
+  } else {
+    auto f = [&](int key, int) {
+      bool ins;
+      probe(K, T - 1, key, ins);
+      cnt += ins;
+    };
+    if (active)
+      for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
+                                          a.vw_log2, f, NoStop{}, long_len);
+    if constexpr (TPR > 32) {
+      if (long_len > 0)
+        for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
+                                             TPR, long_len, s_list, &s_lcnt, f, NoStop{});
     }
   }
   if constexpr (OPT) {
@@ -77,13 +96,14 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
 // on global memory ... set based on the number of intermediate products").
 __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
   __shared__ long long ws[33];
+  __shared__ int s_list[kLongChunk], s_lcnt;
   int* table = a.slab + (long long)blockIdx.x * a.slab_T;
   const long long nA = a.nrows;
   const long long nB = a.dev_count ? (long long)*a.dev_count : 0;
   const int t = threadIdx.x;
   for (long long i = blockIdx.x; i < nA + nB; i += gridDim.x) {
     const int row = i < nA ? a.rows[i] : a.overflow_rows[i - nA];
-    long long cap = a.nprod[row] < a.n ? a.nprod[row] : a.n;
+    const long long cap = a.nprod[row] < a.n ? a.nprod[row] : a.n;
     long long T = 64;
     while (T < 2 * cap) T <<= 1;
     if (T > a.slab_T) T = a.slab_T;
@@ -91,14 +111,17 @@ __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
     for (long long s = t; s < T / 4; s += 1024) t4[s] = make_int4(-1, -1, -1, -1);
     __syncthreads();
     int cnt = 0;
-    const long long a0 = a.a_rpt[row], a1 = a.a_rpt[row + 1];
-    const int vwl = a.vw_log2;
-    const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = 1024 >> vwl;
-    for (long long j = a0 + sub; j < a1; j += nsub) {
-      const int kk = __ldg(a.a_col + j);
-      const long long b0 = __ldg(a.b_rpt + kk), b1 = __ldg(a.b_rpt + kk + 1);
-      for (long long q = b0 + lane; q < b1; q += vw) cnt += hash_insert(table, (unsigned)(T - 1), __ldg(a.b_col + q));
-    }
+    const GKeys K{table};
+    auto f = [&](int key, int) {
+      bool ins;
+      probe(K, (unsigned)(T - 1), key, ins);
+      cnt += ins;
+    };
+    for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, 1024,
+                                        a.vw_log2, f, NoStop{}, a.long_len);
+    if (a.long_len > 0)
+      for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
+                                           a.long_len, s_list, &s_lcnt, f, NoStop{});
     const long long tot = Grp<1024>::sum(cnt, ws);
     if (t == 0) a.c_cnt[row] = tot;
     __syncthreads();

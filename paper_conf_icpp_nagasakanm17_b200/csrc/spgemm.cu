@@ -63,6 +63,7 @@ struct spgemm_ctx {
   bool gtimed[2][kMaxGroups]{};
   // options
   int sym_min_group = -1, num_min_group = -1, fill_limit = 0, use_streams = 1, validate = 0, lanes = 0;
+  int long_len = 0;  // 0 auto, -1 off
   int timing = 1;
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -205,6 +206,13 @@ int auto_vw_log2(spgemm_handle_t h) {
   return l;
 }
 
+// CTA-per-row kernels hand B rows longer than this to the whole CTA (load balance).
+int long_len_of(spgemm_handle_t h) {
+  if (h->long_len < 0) return 0;
+  if (h->long_len > 0) return h->long_len;
+  return std::max(64, 8 << h->vw_log2);
+}
+
 }  // namespace
 
 extern "C" {
@@ -329,6 +337,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       if (v <= 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "budget must be > 0");
       h->ws_budget = v; break;
     case SPGEMM_OPT_TIMING: h->timing = v ? 1 : 0; break;
+    case SPGEMM_OPT_LONG_ROW:
+      if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
+      h->long_len = (int)v; break;
     default: return fail(h, SPGEMM_ERR_INVALID_ARG, "unknown option");
   }
   return SPGEMM_OK;
@@ -419,6 +430,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.a_rpt = a_rpt; sa.a_col = a_col; sa.b_rpt = b_rpt; sa.b_col = b_col;
   sa.c_cnt = c_rpt + 1;
   sa.vw_log2 = h->vw_log2;
+  sa.long_len = long_len_of(h);
   sa.overflow_rows = static_cast<int32_t*>(h->overflow.p);
   sa.overflow_count = &dacc->overflow_count;
   const int T_opt = kSymGroups[kSymOptimistic].T, BS_opt = kSymGroups[kSymOptimistic].BS;
@@ -538,6 +550,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.b_rpt = h->b_rpt; na.b_col = h->b_col; na.b_val = b_val;
     na.c_rpt = h->c_rpt; na.c_col = c_col; na.c_val = c_val;
     na.vw_log2 = h->vw_log2;
+    na.long_len = long_len_of(h);
     na.err_flags = &dacc->err_flags;
     Buf slab;
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
@@ -545,11 +558,13 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     if (n_glob > 0) {
       const long long maxn = std::max<long long>(1, (long long)h->snap2.max_nnz);
       const long long T = std::max<long long>(64, next_pow2(2 * maxn));
-      const long long stride = ((T * vs + T * 4 + (T / 4 + 1) * 4 + maxn * 4) + 255) & ~255LL;
+      const long long words = h->n / 32 + 2;  // bitmap over any column range [lo, hi]
+      const long long stride = ((T * vs + T * 4 + 2 * words * 4) + 255) & ~255LL;
       const long long by_budget = std::max<long long>(1, h->ws_budget / stride);
       glob_grid = (int)std::min<long long>({n_glob, 2LL * h->num_sms, by_budget});
       s = buf_alloc(h, slab, (size_t)(glob_grid * stride));
       if (s != SPGEMM_OK) return s;
+      na.bitmap_words = words;
       na.slab = slab.p; na.slab_T = T; na.slab_stride = stride; na.max_nnz = maxn;
     }
     const int32_t* perm2 = static_cast<const int32_t*>(h->perm2.p);

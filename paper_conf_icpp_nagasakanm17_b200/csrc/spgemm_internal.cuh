@@ -4,8 +4,8 @@
 // Paper map (PAPER.md line numbers):
 //   Alg. 2 n_prod count ........ :90-96   -> k_nprod_group       (kernels_setup.cu)
 //   grouping (2)/(6) ........... :84-88   -> k_group_scatter     (kernels_setup.cu)
-//   Alg. 3/4 thread assignment . :102-126 -> sym_row / num_row   (sub-groups of VW lanes)
-//   Alg. 5 hash insert ......... :130-153 -> hash_insert / hash_slot (below)
+//   Alg. 3/4 thread assignment . :102-126 -> for_each_product    (sub-groups of VW lanes)
+//   Alg. 5 hash insert ......... :130-153 -> probe<SKeys|GKeys> (below)
 //   group-0 overflow retry ..... :155,181 -> optimistic group + k_sym_global
 //   calculation + gather + sort  :171-173 -> num_row (bucket-rank sort)
 //   Table I / parameter rule ... :157-183 -> kSymGroups / kNumGroups (B200 values)
@@ -13,6 +13,8 @@
 
 #include <cuda_runtime.h>
 #include <stdint.h>
+
+#include <climits>
 
 namespace spg {
 
@@ -60,8 +62,8 @@ constexpr int kNumGlobal = 10;
 constexpr int kNumNumGroups = 11;
 
 // Numeric per-row shared-memory layout: vals[T] | keys[T] | bucket[NB+1] | sidx[upper] ,
-// NB = T/4 buckets for the bucket-rank sort.
-__host__ __device__ constexpr int num_nbuckets(int T) { return T / 4; }
+// NB = T/2 (T/4 for the two largest tables) buckets for the bucket-rank sort.
+__host__ __device__ constexpr int num_nbuckets(int T) { return T <= 8192 ? T / 2 : T / 4; }
 __host__ __device__ constexpr int align16(int x) { return (x + 15) & ~15; }
 template <typename VT>
 __host__ __device__ constexpr int num_row_bytes(int T, long long upper) {
@@ -96,35 +98,216 @@ struct Offsets {
 // ----------------------------------------------------------------------------- primitives
 __device__ __forceinline__ int ld_volatile(const int* p) { return *(const volatile int*)p; }
 
-// Algorithm 5: key = col_B[k]; hash = key*HASH_SCAL mod t_size (t_size a
-// power of two -> mask); linear probing; empty = -1; insert by atomicCAS.
-// Returns 1 if this call inserted the key (nz <- nz + 1), else 0.
-__device__ __forceinline__ int hash_insert(int* table, unsigned mask, int key) {
+// Explicit shared-memory access through 32-bit shared-window addresses (keeps the
+// generic->shared conversion out of the hot loops).  No "memory" clobbers: global loads may
+// be scheduled across them; the volatile asm statements keep their mutual order.
+// opaque(): hide a loop-invariant value's derivation so ptxas keeps it in a register instead of
+// rematerialising it (S2R SR_CgaCtaId for shared windows; 64-bit re-association for pointers).
+__device__ __forceinline__ unsigned opaque(unsigned x) { asm volatile("" : "+r"(x)); return x; }
+template <typename T>
+__device__ __forceinline__ T* opaque(T* p) { asm volatile("" : "+l"(p)); return p; }
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return opaque((unsigned)__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ int lds_s32(unsigned a) {
+  int v;
+  asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int cas_s32(unsigned a, int cmp, int val) {
+  int old;
+  asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(a), "r"(cmp), "r"(val));
+  return old;
+}
+__device__ __forceinline__ void red_add_s(unsigned a, float v) { asm volatile("red.shared.add.f32 [%0], %1;" ::"r"(a), "f"(v)); }
+__device__ __forceinline__ void red_add_s(unsigned a, double v) { asm volatile("red.shared.add.f64 [%0], %1;" ::"r"(a), "d"(v)); }
+
+// Key tables in shared (SKeys) or global (GKeys) memory with one probe interface.
+struct SKeys {
+  unsigned base;  // shared address of slot 0
+  __device__ __forceinline__ int ld(unsigned h) const { return lds_s32(base + 4u * h); }
+  __device__ __forceinline__ int cas(unsigned h, int c, int v) const { return cas_s32(base + 4u * h, c, v); }
+};
+struct GKeys {
+  int* p;
+  __device__ __forceinline__ int ld(unsigned h) const { return ld_volatile(p + h); }
+  __device__ __forceinline__ int cas(unsigned h, int c, int v) const { return atomicCAS(p + h, c, v); }
+};
+template <typename VT>
+struct SVals {
+  unsigned base;
+  __device__ __forceinline__ void add(unsigned h, VT v) const { red_add_s(base + (unsigned)sizeof(VT) * h, v); }
+};
+template <typename VT>
+struct GVals {
+  VT* p;
+  __device__ __forceinline__ void add(unsigned h, VT v) const { atomicAdd(p + h, v); }
+};
+
+// Algorithm 5 on either table kind: key = col_B[k]; hash = key*HASH_SCAL
+// mod t_size (t_size a power of two -> mask); linear probing; empty slot = -1;
+// insert by atomicCAS.  Returns the slot of `key`; inserted = this call added it (nz++).
+template <typename Keys>
+__device__ __forceinline__ unsigned probe(const Keys& K, unsigned mask, int key, bool& inserted) {
   unsigned h = ((unsigned)key * kHashScal) & mask;
+  inserted = false;
   while (true) {
-    int cur = ld_volatile(table + h);
-    if (cur == key) return 0;
+    const int cur = K.ld(h);
+    if (cur == key) return h;
     if (cur == -1) {
-      int old = atomicCAS(table + h, -1, key);
-      if (old == -1) return 1;
-      if (old == key) return 0;
+      const int old = K.cas(h, -1, key);
+      if (old == -1) { inserted = true; return h; }
+      if (old == key) return h;
     }
     h = (h + 1) & mask;
   }
 }
 
-// Same probe, returning the slot (numeric phase, "utilizing hash table as well").
-__device__ __forceinline__ unsigned hash_slot(int* table, unsigned mask, int key, bool& inserted) {
-  unsigned h = ((unsigned)key * kHashScal) & mask;
+// Iterate the intermediate products of one row (Alg. 3/4 loops generalised): sub-groups of
+// VW lanes walk the row's A non-zeros, lanes stride VW over each B row.  Two-stage software
+// pipeline over A non-zeros: while B row j is processed, rpt_B of j+1 and col_A of j+2 are
+// already in flight; B rows are unrolled by 2 so each lane has two gathers outstanding.
+// f(key, value) is called per product; stop() (checked per product when CHECK_STOP) aborts.
+// Load balance (CTA-per-row groups): with long_len > 0 a sub-group skips B rows longer than
+// long_len; the caller then runs for_long_products, where the whole CTA walks each of them
+// (hub columns of power-law graphs would otherwise serialise a CTA behind one sub-group).
+template <bool NUM, bool CHECK_STOP, typename VT, typename F, typename S>
+__device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
+                                                 const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
+                                                 const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
+                                                 int row, int t, int tpr, int vwl, F&& f, S&& stop,
+                                                 int long_len = 0) {
+  const long long a0 = __ldg(a_rpt + row);
+  const int na = (int)(__ldg(a_rpt + row + 1) - a0);  // row-relative 32-bit indexing
+  const int32_t* __restrict__ ac = opaque(a_col + a0);
+  const VT* __restrict__ avp = NUM ? opaque(a_val + a0) : nullptr;
+  const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = tpr >> vwl;
+  int j = sub;
+  if (j >= na) return;
+  int kk = __ldg(ac + j);
+  VT av = NUM ? __ldg(avp + j) : VT(0);
+  int jn = j + nsub;
+  int kkn = 0;
+  VT avn = VT(0);
+  if (jn < na) { kkn = __ldg(ac + jn); if (NUM) avn = __ldg(avp + jn); }
+  long long b0 = __ldg(b_rpt + kk);
+  int len = (int)(__ldg(b_rpt + kk + 1) - b0);
   while (true) {
-    int cur = ld_volatile(table + h);
-    if (cur == key) { inserted = false; return h; }
-    if (cur == -1) {
-      int old = atomicCAS(table + h, -1, key);
-      if (old == -1) { inserted = true; return h; }
-      if (old == key) { inserted = false; return h; }
+    long long b0n = 0;
+    int lenn = 0;
+    if (jn < na) { b0n = __ldg(b_rpt + kkn); lenn = (int)(__ldg(b_rpt + kkn + 1) - b0n); }
+    const int jnn = jn + nsub;
+    int kknn = 0;
+    VT avnn = VT(0);
+    if (jnn < na) { kknn = __ldg(ac + jnn); if (NUM) avnn = __ldg(avp + jnn); }
+    const int32_t* __restrict__ bc = opaque(b_col + b0);
+    const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
+    if (long_len > 0 && len > long_len) len = 0;  // deferred to for_long_products
+#pragma unroll 1
+    for (int q = lane; q < len; q += 2 * vw) {
+      const int k0 = __ldg(bc + q);
+      const VT v0 = NUM ? __ldg(bv + q) : VT(0);
+      const bool h1 = q + vw < len;
+      int k1 = 0;
+      VT v1 = VT(0);
+      if (h1) { k1 = __ldg(bc + q + vw); if (NUM) v1 = __ldg(bv + q + vw); }
+      if (CHECK_STOP && stop()) return;
+      f(k0, av * v0);
+      if (h1) {
+        if (CHECK_STOP && stop()) return;
+        f(k1, av * v1);
+      }
     }
-    h = (h + 1) & mask;
+    if (jn >= na) return;
+    if (CHECK_STOP && stop()) return;
+    j = jn;
+    kk = kkn; av = avn; b0 = b0n; len = lenn;
+    jn = jnn; kkn = kknn; avn = avnn;
+  }
+}
+
+// Second pass (CTA-wide, every thread of the CTA must call it): the A row is rescanned in
+// chunks of kLongChunk entries; entries whose B row is longer than long_len go to a shared
+// list, and all tpr threads stride each listed B row (unrolled by 2).  s_list: kLongChunk
+// ints, s_cnt: one int, both shared.  A stopped (CHECK_STOP) thread keeps hitting barriers.
+constexpr int kLongChunk = 256;
+template <bool NUM, bool CHECK_STOP, typename VT, typename F, typename S>
+__device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
+                                                  const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
+                                                  const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
+                                                  bool active, int row, int t, int tpr, int long_len, int* s_list,
+                                                  int* s_cnt, F&& f, S&& stop) {
+  const long long a0 = active ? __ldg(a_rpt + row) : 0;
+  const int na = active ? (int)(__ldg(a_rpt + row + 1) - a0) : 0;
+  const int32_t* __restrict__ ac = a_col + a0;
+  if (t == 0) *s_cnt = 0;
+  __syncthreads();
+  for (int c = 0; c < na; c += kLongChunk) {  // na is CTA-uniform
+    for (int e = t; e < kLongChunk && c + e < na; e += tpr) {
+      const int kk = __ldg(ac + c + e);
+      if (__ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk) > long_len) s_list[atomicAdd(s_cnt, 1)] = c + e;
+    }
+    __syncthreads();
+    const int n = *s_cnt;
+    for (int i = 0; i < n; ++i) {
+      const int j = s_list[i];
+      const int kk = __ldg(ac + j);
+      const VT av = NUM ? __ldg(a_val + a0 + j) : VT(0);
+      const long long b0 = __ldg(b_rpt + kk);
+      int len = (int)(__ldg(b_rpt + kk + 1) - b0);
+      if (CHECK_STOP && stop()) len = 0;
+      const int32_t* __restrict__ bc = opaque(b_col + b0);
+      const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
+#pragma unroll 1
+      for (int q = t; q < len; q += 2 * tpr) {
+        const int k0 = __ldg(bc + q);
+        const VT v0 = NUM ? __ldg(bv + q) : VT(0);
+        const bool h1 = q + tpr < len;
+        int k1 = 0;
+        VT v1 = VT(0);
+        if (h1) { k1 = __ldg(bc + q + tpr); if (NUM) v1 = __ldg(bv + q + tpr); }
+        if (CHECK_STOP && stop()) break;
+        f(k0, av * v0);
+        if (h1) {
+          if (CHECK_STOP && stop()) break;
+          f(k1, av * v1);
+        }
+      }
+    }
+    __syncthreads();
+    if (t == 0) *s_cnt = 0;
+    __syncthreads();
+  }
+}
+
+// Warp-aggregated per-group accumulation into shared counters (64-bit shared atomics are
+// CAS loops on sm_100a, so each distinct group of the warp issues one atomic per counter).
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  return x;
+}
+__device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long y = __shfl_xor_sync(0xffffffffu, x, o);
+    x = y > x ? y : x;
+  }
+  return x;
+}
+template <int NV>
+__device__ __forceinline__ void warp_group_add(bool valid, int g, const unsigned long long (&v)[NV],
+                                               unsigned long long* const (&dst)[NV]) {
+  const int lane = threadIdx.x & 31;
+  unsigned todo = __ballot_sync(0xffffffffu, valid);
+  while (todo) {
+    const int leader = __ffs(todo) - 1;
+    const int gl = __shfl_sync(0xffffffffu, g, leader);
+    const bool mine = valid && g == gl;
+    todo &= ~__ballot_sync(0xffffffffu, mine);
+#pragma unroll
+    for (int i = 0; i < NV; ++i) {
+      const unsigned long long x = warp_sum_u64(mine ? v[i] : 0ull);
+      if (lane == leader) atomicAdd(dst[i] + gl, x);
+    }
   }
 }
 
@@ -132,8 +315,13 @@ __device__ __forceinline__ unsigned hash_slot(int* table, unsigned mask, int key
 // TPR > 32 -> the whole CTA (one row per CTA), ws = >= 33 ints of shared scratch.
 template <int TPR>
 struct Grp {
+  // lanes of this row group inside its warp (TPR < 32), so rows sharing a warp may diverge
+  static __device__ __forceinline__ unsigned mask() {
+    if constexpr (TPR >= 32) return 0xffffffffu;
+    else return ((1u << TPR) - 1u) << ((threadIdx.x & 31) & ~(TPR - 1));
+  }
   static __device__ __forceinline__ void sync() {
-    if constexpr (TPR <= 32) __syncwarp(); else __syncthreads();
+    if constexpr (TPR <= 32) __syncwarp(mask()); else __syncthreads();
   }
   static __device__ __forceinline__ int lane() { return threadIdx.x % TPR; }
 
@@ -143,10 +331,10 @@ struct Grp {
       long long x = v;
 #pragma unroll
       for (int d = 1; d < TPR; d <<= 1) {
-        long long y = __shfl_up_sync(0xffffffffu, x, d, TPR);
+        long long y = __shfl_up_sync(mask(), x, d, TPR);
         if (lane() >= d) x += y;
       }
-      *total = __shfl_sync(0xffffffffu, x, TPR - 1, TPR);
+      *total = __shfl_sync(mask(), x, TPR - 1, TPR);
       return x - v;
     } else {
       constexpr int NW = TPR / 32;
@@ -176,6 +364,30 @@ struct Grp {
     }
   }
 
+  // group min of mn and max of mx, written to out[0], out[1] (visible to the whole group on
+  // return); out must be per-group shared memory.
+  static __device__ __forceinline__ void minmax(int mn, int mx, int* out) {
+    if constexpr (TPR <= 32) {
+#pragma unroll
+      for (int o = TPR / 2; o > 0; o >>= 1) {
+        mn = min(mn, __shfl_xor_sync(mask(), mn, o, TPR));
+        mx = max(mx, __shfl_xor_sync(mask(), mx, o, TPR));
+      }
+      if (lane() == 0) { out[0] = mn; out[1] = mx; }
+      __syncwarp(mask());
+    } else {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+      }
+      if (threadIdx.x == 0) { out[0] = INT_MAX; out[1] = -1; }
+      __syncthreads();
+      if ((threadIdx.x & 31) == 0) { atomicMin(out, mn); atomicMax(out + 1, mx); }
+      __syncthreads();
+    }
+  }
+
   static __device__ __forceinline__ long long sum(long long v, long long* ws) {
     long long t;
     excl_scan(v, &t, ws);
@@ -191,6 +403,7 @@ struct SymArgs {
   long long nrows;
   int64_t* c_cnt;          // c_rpt + 1: per-row nnz written here (scanned later)
   int vw_log2;             // lanes per B row = 1 << vw_log2 (Alg. 3/4 generalised)
+  int long_len;            // CTA-per-row groups: B rows longer than this are walked by the CTA
   // optimistic group
   int32_t* overflow_rows; int* overflow_count; int fill_limit;
   // global fallback
@@ -204,9 +417,10 @@ struct NumArgs {
   const int32_t* rows; long long nrows;
   const int64_t* c_rpt; int32_t* c_col; void* c_val;
   int vw_log2;
+  int long_len;
   int* err_flags;
   // global fallback
-  void* slab; long long slab_T; long long slab_stride; long long max_nnz;
+  void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;
 };
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,

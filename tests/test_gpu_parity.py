@@ -152,6 +152,18 @@ def test_lanes_per_b_row(spg, lanes):
     assert_parity(got, ref, np.float64, exact=True, what=f"lanes={lanes}")
 
 
+@pytest.mark.parametrize("long_row", [-1, 1, 16])
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_long_row_cta_pass(spg, long_row, dtype):
+    """B rows longer than long_row are walked by the whole CTA (second pass); 1 = every row."""
+    A = _mixed_small()
+    ref = oracle.spgemm(A.astype(dtype), A.astype(dtype), dtype)
+    for opts in ({"long_row": long_row}, {"long_row": long_row, "sym_min_group": 10, "sym_fill_limit": 64},
+                 {"long_row": long_row, "sym_min_group": 11, "num_min_group": 10}):
+        got = run_gpu(spg, A, A, dtype, opts)
+        assert_parity(got, ref, dtype, what=f"{opts}")
+
+
 def test_serial_streams(spg):
     A = _mixed_small()
     ref = oracle.spgemm(A, A, np.float64)
