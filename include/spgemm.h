@@ -22,7 +22,8 @@
  *
  * Ownership: the caller owns A, B and all of C.  The library owns only its workspace
  * (grouping arrays, n_prod, global-memory hash tables), obtained from the allocator given to
- * spgemm_create (NULL -> cudaMallocAsync on the handle's stream).  A's and B's structure
+ * spgemm_create (NULL -> a private stream-ordered CUDA memory pool of the handle whose
+ * memory stays mapped between calls and is released by spgemm_destroy).  A's and B's structure
  * arrays are BORROWED from spgemm_symbolic until the next spgemm_symbolic/destroy: they
  * must stay alive and unchanged while spgemm_numeric may be called (structure reuse).
  *
@@ -123,8 +124,11 @@ typedef enum {
     SPGEMM_OPT_LANES = 5,           /* lanes per B row (power of two 1..32), 0 = auto */
     SPGEMM_OPT_WORKSPACE_BUDGET = 6,/* max bytes for global-memory hash tables */
     SPGEMM_OPT_TIMING = 7,          /* 1 = per-group CUDA-event timing (default 1) */
-    SPGEMM_OPT_LONG_ROW = 8         /* CTA-per-row groups: B rows longer than v are walked by
+    SPGEMM_OPT_LONG_ROW = 8,        /* CTA-per-row groups: B rows longer than v are walked by
                                        the whole CTA (0 = auto, -1 = off) */
+    SPGEMM_OPT_RANGE_HASH = 9       /* 1 (default): rows whose column span fits the group's table
+                                       use the offset hash key - lo_i (collision-free, ordered);
+                                       0: the paper's multiplicative hash (Alg. 5) everywhere */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

@@ -23,7 +23,7 @@ STATUS = {
 
 OPTIONS = {
     "sym_min_group": 0, "num_min_group": 1, "sym_fill_limit": 2, "streams": 3,
-    "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8,
+    "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8, "range_hash": 9,
 }
 
 # Symbols declared in include/spgemm.h (tests check the .so exports all of them).

@@ -13,7 +13,9 @@
 //   (c1) range/NB <= 4 (banded/FEM rows): entries are scattered into NB buckets of width
 //        <= 4 and rank = bucket start + #smaller keys in the bucket (the paper's comparison
 //        rank restricted to a bucket) — a prefix count when the range fits NB;
-//   (c2) wider ranges in shared memory: bitonic sort of the compacted slot indices;
+//   (c4) wider ranges, CTA-per-row groups: same buckets, then one warp per bucket ranks its
+//        keys by shuffle comparisons (<= 32 keys) or a per-warp bitmap + popcount prefix;
+//   (c2) wider ranges, sub-warp row groups (<= 128 keys): bitonic sort of the slot indices;
 //   (c3) global-memory rows: bitmap over [lo, hi] + prefix popcounts.
 // Keys are distinct, so every path writes the identical, sorted row.
 #include <climits>
@@ -23,6 +25,11 @@
 namespace spg {
 
 namespace {
+
+// bitmap words per warp for the (c4) rank: 4096 columns for small CTAs, 1024 for 512/1024
+// threads (shared memory of the largest tables).
+template <int TPR>
+constexpr int kWarpBitmapWords = TPR <= 256 ? 128 : 32;
 
 struct NoStop {
   __device__ __forceinline__ bool operator()() const { return false; }
@@ -40,9 +47,71 @@ struct Vec16<double> { using T = double2; static __device__ __forceinline__ doub
 template <typename VT, int TPR, bool GLOBAL, typename Keys, typename Vals, typename SIdx>
 __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, const Keys& K, const Vals& V,
                                         int* Kp, VT* Vp, int* Bc, SIdx* S, unsigned mask, int NB, int* lohi,
-                                        long long* ws, int* s_list, int* s_lcnt) {
+                                        long long* ws, int* s_list, int* s_lcnt, unsigned* wscr) {
   const int t = Grp<TPR>::lane();
   const unsigned T = mask + 1;
+  if (TPR > 32 && t == 0) *s_lcnt = 0;  // pass-1 "deferred a long row" flag (read after a barrier)
+  if constexpr (!GLOBAL) {
+    // Range-offset hash: when the row's column span R fits the table, slot =
+    // key - lo_i (collision-free, order-preserving).  Vp[0..R) accumulates; the bytes of
+    // Kp[0..R/4) flag occupancy (plain idempotent stores; structural zeros stay); the gather is
+    // an in-order compaction of the flags.
+    if (active && a.rlohi != nullptr) {
+      const int2 rr = __ldg(a.rlohi + row);
+      const long long R = (long long)rr.y - rr.x + 1;
+      if (R > 0 && R <= (long long)T) {  // uniform within the row group
+        const int lo = rr.x;
+        const int words = (int)((R + 3) >> 2);  // 4 flag bytes per word
+        using V16 = typename Vec16<VT>::T;
+        constexpr int per = 16 / sizeof(VT);
+        V16* v16 = reinterpret_cast<V16*>(Vp);
+        for (int s = t; s < (int)((R + per - 1) / per); s += TPR) v16[s] = Vec16<VT>::zero();
+        int4* k4 = reinterpret_cast<int4*>(Kp);
+        for (int s = t; s < (words + 3) / 4; s += TPR) k4[s] = make_int4(0, 0, 0, 0);
+        Grp<TPR>::sync();
+        const unsigned kb = smem_u32(Kp);
+        auto f = [&](int key, VT prod) {
+          const unsigned d = (unsigned)(key - lo);
+          st_s8(kb + d, 1);
+          V.add(d, prod);
+        };
+        const int long_len = TPR > 32 ? a.long_len : 0;
+        for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
+                                          static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
+                                          long_len, s_lcnt);
+        if constexpr (TPR > 32) {
+          if (long_len > 0)
+            for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
+                                               a.b_col, static_cast<const VT*>(a.b_val), true, row, t, TPR,
+                                               long_len, s_list, s_lcnt, f, NoStop{});
+        }
+        Grp<TPR>::sync();
+        // in-order compaction: thread owns a contiguous run of flag words
+        const int pw = (words + TPR - 1) / TPR;
+        const int w0 = t * pw, w1 = min(words, w0 + pw);
+        long long loc = 0;
+        for (int w = w0; w < w1; ++w) loc += __popc((unsigned)Kp[w]);
+        long long n_total;
+        long long r = Grp<TPR>::excl_scan(loc, &n_total, ws);
+        const long long c0 = a.c_rpt[row];
+        const long long cn = a.c_rpt[row + 1] - c0;
+        if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
+        VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+        int32_t* __restrict__ cc = a.c_col + c0;
+        for (int w = w0; w < w1; ++w) {
+          unsigned bits = (unsigned)Kp[w];
+          while (bits) {
+            const int d = w * 4 + ((__ffs(bits) - 1) >> 3);
+            bits &= bits - 1;
+            if (r < cn) { cc[r] = lo + d; cv[r] = Vp[d]; }
+            ++r;
+          }
+        }
+        Grp<TPR>::sync();
+        return;
+      }
+    }
+  }
   // (0) keys <- -1 (Alg. 5 precondition), values <- 0; 16-byte stores
   {
     int4* k4 = reinterpret_cast<int4*>(Kp);
@@ -65,7 +134,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
     if (active)
       for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
                                         static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
-                                        long_len);
+                                        long_len, s_lcnt);
     if constexpr (TPR > 32) {
       if (long_len > 0)
         for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
@@ -134,11 +203,14 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
     if (hi >= lo) {
       const unsigned R = (unsigned)(hi - lo);
       while ((R >> shift) >= (unsigned)NB) ++shift;
+      // (c4) ranks dense buckets with a per-warp bitmap of 32*kWarpBitmapWords columns, so
+      // wide buckets cost nothing extra there while empty buckets cost a warp visit each.
+      if (TPR > 32 && shift > 2 && shift < 10) shift = 10;
       nb = (int)(R >> shift) + 1;
     }
-    if (shift <= 2) {
-      // (c1) bucket rank: NB buckets of width 2^shift <= 4 over [lo, hi]; rank = bucket start
-      // + #smaller keys in the same bucket (the paper's comparison rank, within a bucket).
+    if (shift <= 2 || TPR > 32) {
+      // Buckets of width 2^shift over [lo, hi]: histogram, exclusive scan, scatter of the
+      // slot indices into bucket order (Bc[b] = start of bucket b afterwards).
       for (int b = t; b <= nb; b += TPR) Bc[b] = 0;
       Grp<TPR>::sync();
       for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
@@ -168,16 +240,80 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
         if (kv.w >= 0) S[atomicAdd(&Bc[1 + ((kv.w - lo) >> shift)], 1)] = (SIdx)(s + 3);
       }
       Grp<TPR>::sync();
-      if (active) {
-        if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
-        for (int p = t; p < (int)n_total; p += TPR) {
-          const unsigned s = S[p];
-          const int key = Kp[s];
-          const int b = (key - lo) >> shift;
-          const int st = Bc[b], en = Bc[b + 1];
-          int r = st;
-          for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
-          if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
+      if (t == 0 && active && cn != n_total) atomicOr(a.err_flags, 2);
+      if (shift <= 2) {
+        // (c1) rank = bucket start + #smaller keys in the bucket (<= 4 keys per bucket)
+        if (active) {
+          for (int p = t; p < (int)n_total; p += TPR) {
+            const unsigned s = S[p];
+            const int key = Kp[s];
+            const int b = (key - lo) >> shift;
+            const int st = Bc[b], en = Bc[b + 1];
+            int r = st;
+            for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
+            if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
+          }
+        }
+      } else if constexpr (TPR > 32) {
+        // (c4) one warp per bucket: <= 32 keys -> rank by shuffle comparisons; denser buckets
+        // of width <= 1024 -> per-warp bitmap + popcount prefix; wider -> comparisons.
+        constexpr int MW = kWarpBitmapWords<TPR>;  // bitmap words per warp (32 per 1024 columns)
+        constexpr int WPL = MW / 32;
+        const int wid = t >> 5, ln = t & 31;
+        unsigned* wb = wscr + wid * 2 * MW;
+        unsigned* wp = wb + MW;
+        const int words = (int)(((1u << shift) + 31) >> 5);
+        for (int b = wid; b < nb; b += TPR / 32) {
+          const int st = Bc[b], en = Bc[b + 1], c = en - st;  // warp-uniform
+          if (c == 0 || !active) continue;
+          const int base = lo + (b << shift);
+          if (c <= 32) {
+            const unsigned slot = ln < c ? (unsigned)S[st + ln] : 0u;
+            const int key = ln < c ? Kp[slot] : INT_MAX;
+            int r = 0;
+            for (int m = 0; m < c; ++m) r += __shfl_sync(0xffffffffu, key, m) < key;
+            if (ln < c && st + r < cn) { cc[st + r] = key; cv[st + r] = Vp[slot]; }
+          } else if (words <= MW) {
+            for (int w = ln; w < words; w += 32) wb[w] = 0u;
+            __syncwarp();
+            for (int p = st + ln; p < en; p += 32) {
+              const unsigned d = (unsigned)(Kp[S[p]] - base);
+              atomicOr(wb + (d >> 5), 1u << (d & 31));
+            }
+            __syncwarp();
+            unsigned loc[WPL], sum = 0;
+#pragma unroll
+            for (int u = 0; u < WPL; ++u) {
+              loc[u] = ln * WPL + u < words ? __popc(wb[ln * WPL + u]) : 0u;
+              sum += loc[u];
+            }
+            unsigned incl = sum;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+              const unsigned y = __shfl_up_sync(0xffffffffu, incl, o);
+              if (ln >= o) incl += y;
+            }
+            unsigned ex = incl - sum;
+#pragma unroll
+            for (int u = 0; u < WPL; ++u) { wp[ln * WPL + u] = ex; ex += loc[u]; }
+            __syncwarp();
+            for (int p = st + ln; p < en; p += 32) {
+              const unsigned slot = S[p];
+              const int key = Kp[slot];
+              const unsigned d = (unsigned)(key - base);
+              const int r = st + (int)wp[d >> 5] + __popc(wb[d >> 5] & ((1u << (d & 31)) - 1u));
+              if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
+            }
+            __syncwarp();
+          } else {
+            for (int p = st + ln; p < en; p += 32) {
+              const unsigned slot = S[p];
+              const int key = Kp[slot];
+              int r = st;
+              for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
+              if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
+            }
+          }
         }
       }
     } else {
@@ -238,6 +374,7 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   constexpr int RPB = BS / TPR;
   __shared__ int s_lohi[2 * RPB];
   __shared__ int s_list[TPR > 32 ? kLongChunk : 1], s_lcnt;
+  __shared__ unsigned s_wscr[TPR > 32 ? (TPR / 32) * 2 * kWarpBitmapWords<TPR> : 1];  // bucket bitmap+prefix
   constexpr int NB = num_nbuckets(T);
   constexpr int RB = num_row_bytes<VT>(T, UPPER);
   const int g = threadIdx.x / TPR;
@@ -250,7 +387,7 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : 0;
   num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
-                   s_lohi + 2 * g, ws, s_list, &s_lcnt);
+                   s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr);
 }
 
 template <typename VT>
@@ -270,7 +407,7 @@ __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
     while (T < 2 * n) T <<= 1;
     if (T > a.slab_T) T = a.slab_T;
     num_row<VT, 1024, true>(a, true, row, GKeys{Kp}, GVals<VT>{Vp}, Kp, Vp, Bc, S, (unsigned)(T - 1), 0,
-                      s_lohi, ws, s_list, &s_lcnt);
+                      s_lohi, ws, s_list, &s_lcnt, nullptr);
   }
 }
 
@@ -278,7 +415,8 @@ template <typename VT, int T, int TPR, int BS, long long UPPER>
 cudaError_t launch_num(cudaStream_t s, const NumArgs& a) {
   constexpr int RPB = BS / TPR;
   constexpr int smem = RPB * num_row_bytes<VT>(T, UPPER);
-  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 <= kSmemLimit, "numeric table too large");
+  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 + (TPR > 32 ? TPR / 32 * 8 * kWarpBitmapWords<TPR> : 4) <= kSmemLimit,
+                "numeric table too large");
   static bool configured = false;
   if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(k_num_smem<VT, T, TPR, BS, UPPER>,

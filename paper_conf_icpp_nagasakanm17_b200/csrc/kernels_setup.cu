@@ -8,6 +8,8 @@
 //                   the first kernel fused with the step-(6) grouping by nnz_i.
 //   k_validate      optional O(nnz) input validation.
 //   k_splits        n_prod-balanced row blocks for the multi-GPU driver.
+#include <climits>
+
 #include "spgemm_internal.cuh"
 
 namespace spg {
@@ -23,55 +25,119 @@ __device__ __forceinline__ int group_of(long long key, const Bounds& bd) {
   return g;
 }
 
-template <int LPR>
+// Per-group row counts with warp-aggregated 32-bit shared atomics (MATCH.ANY on the group).
+__device__ __forceinline__ void count_group(bool valid, int g, int* s_cnt) {
+  const unsigned peers = __match_any_sync(0xffffffffu, valid ? g : -1);
+  const int lane = threadIdx.x & 31;
+  if (valid && lane == __ffs(peers) - 1) atomicAdd(&s_cnt[g], __popc(peers));
+}
+
+// Column range of every B row: bmm[k] = {min col, max col} ({INT_MAX, -1} if empty).  One
+// row per thread; rows longer than kLongA entries are reduced by the whole warp.
+constexpr int kLongA = 16;
+__global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, const int64_t* __restrict__ b_rpt,
+                                                               const int32_t* __restrict__ b_col,
+                                                               int2* __restrict__ bmm) {
+  const int lane = threadIdx.x & 31;
+  const long long row = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
+  long long b0 = 0, b1 = 0;
+  if (row < k) { b0 = b_rpt[row]; b1 = b_rpt[row + 1]; }
+  const bool is_long = b1 - b0 > kLongA;
+  int mn = INT_MAX, mx = -1;
+  if (!is_long)
+    for (long long j = b0; j < b1; ++j) {
+      const int c = __ldg(b_col + j);
+      mn = min(mn, c); mx = max(mx, c);
+    }
+  unsigned longs = __ballot_sync(0xffffffffu, is_long);
+  while (longs) {
+    const int src = __ffs(longs) - 1;
+    longs &= longs - 1;
+    const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
+    int pmn = INT_MAX, pmx = -1;
+    for (long long j = s0 + lane; j < s1; j += 32) {
+      const int c = __ldg(b_col + j);
+      pmn = min(pmn, c); pmx = max(pmx, c);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
+      pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
+    }
+    if (lane == src) { mn = pmn; mx = pmx; }
+  }
+  if (row < k) bmm[row] = make_int2(mn, mx);
+}
+
+// One row per thread; rows longer than kLongA entries are summed by the whole warp
+// (coalesced), so power-law rows do not serialise a warp behind one thread.  Also the column
+// span [lo_i, hi_i] of row i of C (min/max over its A entries of the B-row ranges): exact,
+// since every B column appears in C (kept structurally).
 __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
     long long m, const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
-    const int64_t* __restrict__ b_rpt, int64_t* __restrict__ nprod, uint8_t* __restrict__ grp,
-    int64_t* __restrict__ c_rpt, DevAcc* __restrict__ acc, Bounds bd) {
-  __shared__ unsigned long long s_rows[kMaxGroups], s_np[kMaxGroups], s_nza[kMaxGroups];
+    const int64_t* __restrict__ b_rpt, const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
+    int2* __restrict__ rlohi, uint8_t* __restrict__ grp, int64_t* __restrict__ c_rpt,
+    DevAcc* __restrict__ acc, Bounds bd) {
+  __shared__ int s_cnt[kMaxGroups];
   __shared__ unsigned long long s_total, s_max;
-  if (threadIdx.x < kMaxGroups) {
-    s_rows[threadIdx.x] = 0; s_np[threadIdx.x] = 0; s_nza[threadIdx.x] = 0;
-  }
+  if (threadIdx.x < kMaxGroups) s_cnt[threadIdx.x] = 0;
   if (threadIdx.x == 0) { s_total = 0; s_max = 0; }
   __syncthreads();
-  constexpr int RPB = kSetupThreads / LPR;
-  const long long row = (long long)blockIdx.x * RPB + threadIdx.x / LPR;
-  const int l = threadIdx.x % LPR;
-  long long np = 0, a0 = 0, a1 = 0;
-  if (row < m) {
-    a0 = a_rpt[row];
-    a1 = a_rpt[row + 1];
-    // Alg. 2: n_prod += rpt_B[col_A[j]+1] - rpt_B[col_A[j]], j in [rpt_A[i], rpt_A[i+1])
-    for (long long j = a0 + l; j < a1; j += LPR) {
-      const int kk = __ldg(a_col + j);
-      np += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
+  const int lane = threadIdx.x & 31;
+  const long long row = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
+  long long a0 = 0, a1 = 0;
+  if (row < m) { a0 = a_rpt[row]; a1 = a_rpt[row + 1]; }
+  const bool is_long = a1 - a0 > kLongA;
+  // Alg. 2: n_prod += rpt_B[col_A[j]+1] - rpt_B[col_A[j]], j in [rpt_A[i], rpt_A[i+1])
+  long long np = 0;
+  int lo = INT_MAX, hi = -1;
+  if (!is_long) {  // <= kLongA entries: issue the col_A loads, then the rpt_B gathers, 4 at a time
+    for (long long j = a0; j < a1; j += 4) {
+      int kk[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) kk[u] = j + u < a1 ? __ldg(a_col + j + u) : -1;
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (kk[u] >= 0) {
+          np += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+          if (bmm) { const int2 r = __ldg(bmm + kk[u]); lo = min(lo, r.x); hi = max(hi, r.y); }
+        }
     }
   }
+  unsigned longs = __ballot_sync(0xffffffffu, is_long);
+  while (longs) {
+    const int src = __ffs(longs) - 1;
+    longs &= longs - 1;
+    const long long s0 = __shfl_sync(0xffffffffu, a0, src), s1 = __shfl_sync(0xffffffffu, a1, src);
+    long long part = 0;
+    int plo = INT_MAX, phi = -1;
+    for (long long j = s0 + lane; j < s1; j += 32) {
+      const int kk = __ldg(a_col + j);
+      part += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
+      if (bmm) { const int2 r = __ldg(bmm + kk); plo = min(plo, r.x); phi = max(phi, r.y); }
+    }
+    part = (long long)warp_sum_u64((unsigned long long)part);
 #pragma unroll
-  for (int off = LPR / 2; off > 0; off >>= 1) np += __shfl_xor_sync(0xffffffffu, np, off);
-  int g = 0xFF;
-  const bool lead = row < m && l == 0;
-  if (lead) {
+    for (int o = 16; o > 0; o >>= 1) {
+      plo = min(plo, __shfl_xor_sync(0xffffffffu, plo, o));
+      phi = max(phi, __shfl_xor_sync(0xffffffffu, phi, o));
+    }
+    if (lane == src) { np = part; lo = plo; hi = phi; }
+  }
+  int g = -1;
+  if (row < m) {
     nprod[row] = np;
+    if (rlohi) rlohi[row] = make_int2(lo, hi);
     if (np == 0) c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
     else g = group_of(np, bd);
-    grp[row] = (uint8_t)g;
+    grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
   }
-  {
-    const unsigned long long v[3] = {1ull, (unsigned long long)np, (unsigned long long)(a1 - a0)};
-    unsigned long long* const d[3] = {s_rows, s_np, s_nza};
-    warp_group_add<3>(lead && g != 0xFF, g, v, d);
-    const unsigned long long tot = warp_sum_u64(lead ? (unsigned long long)np : 0ull);
-    const unsigned long long mx = warp_max_u64(lead ? (unsigned long long)np : 0ull);
-    if ((threadIdx.x & 31) == 0) { atomicAdd(&s_total, tot); atomicMax(&s_max, mx); }
-  }
+  count_group(g >= 0, g, s_cnt);
+  const unsigned long long tot = warp_sum_u64((unsigned long long)np);
+  const unsigned long long mx = warp_max_u64((unsigned long long)np);
+  if (lane == 0) { atomicAdd(&s_total, tot); atomicMax(&s_max, mx); }
   __syncthreads();
-  if (threadIdx.x < kMaxGroups && s_rows[threadIdx.x]) {
-    atomicAdd(&acc->sym_rows[threadIdx.x], s_rows[threadIdx.x]);
-    atomicAdd(&acc->sym_nprod[threadIdx.x], s_np[threadIdx.x]);
-    atomicAdd(&acc->sym_nnza[threadIdx.x], s_nza[threadIdx.x]);
-  }
+  if (threadIdx.x < kMaxGroups && s_cnt[threadIdx.x]) atomicAdd(&acc->sym_rows[threadIdx.x], (unsigned long long)s_cnt[threadIdx.x]);
   if (threadIdx.x == 0) {
     atomicAdd(&acc->total_nprod, s_total);
     atomicMax(&acc->max_nprod, s_max);
@@ -119,56 +185,89 @@ __device__ __forceinline__ long long block_sum_ll(long long v, long long* ws) {
   return Grp<kSetupThreads>::sum(v, ws);
 }
 
-// Tile reduction of x[0..m) (x = rpt_C + 1 holding nnz_i), fused with grouping by nnz_i.
-__global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(
-    long long m, const int64_t* __restrict__ x, long long* __restrict__ tile_sums,
-    const int64_t* __restrict__ nprod, const int64_t* __restrict__ a_rpt, uint8_t* __restrict__ grp2,
-    DevAcc* __restrict__ acc, Bounds bd) {
+// Tile reduction of x[0..m) (x = rpt_C + 1 holding nnz_i), fused with grouping by nnz_i
+// (group ids, per-group row counts and the maximum nnz_i: what the host needs at sync 2).
+__global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(long long m, const int64_t* __restrict__ x,
+                                                               long long* __restrict__ tile_sums,
+                                                               uint8_t* __restrict__ grp2, DevAcc* __restrict__ acc,
+                                                               Bounds bd) {
   __shared__ long long ws[33];
-  __shared__ unsigned long long s_rows[kMaxGroups], s_np[kMaxGroups], s_nza[kMaxGroups], s_nzc[kMaxGroups];
+  __shared__ int s_cnt[kMaxGroups];
   __shared__ unsigned long long s_max;
   const bool grouping = grp2 != nullptr;
   if (grouping) {
-    if (threadIdx.x < kMaxGroups) {
-      s_rows[threadIdx.x] = 0; s_np[threadIdx.x] = 0; s_nza[threadIdx.x] = 0; s_nzc[threadIdx.x] = 0;
-    }
+    if (threadIdx.x < kMaxGroups) s_cnt[threadIdx.x] = 0;
     if (threadIdx.x == 0) s_max = 0;
     __syncthreads();
   }
   const long long base = (long long)blockIdx.x * kScanTile;
   long long s = 0;
+  unsigned long long mx = 0;
 #pragma unroll
   for (int e = 0; e < kScanItems; ++e) {
     const long long i = base + e * kSetupThreads + threadIdx.x;
     const long long v = i < m ? x[i] : 0;
     s += v;
     if (grouping) {  // block-uniform branch
-      int g = 0xFF;
+      int g = -1;
       if (i < m) {
         if (v > 0) g = group_of(v, bd);
-        grp2[i] = (uint8_t)g;
+        grp2[i] = (uint8_t)(g < 0 ? 0xFF : g);
       }
-      const bool valid = g != 0xFF;
-      const unsigned long long vv[4] = {1ull, (unsigned long long)v,
-                                        valid ? (unsigned long long)nprod[i] : 0ull,
-                                        valid ? (unsigned long long)(a_rpt[i + 1] - a_rpt[i]) : 0ull};
-      unsigned long long* const d[4] = {s_rows, s_nzc, s_np, s_nza};
-      warp_group_add<4>(valid, g, vv, d);
-      const unsigned long long mx = warp_max_u64(valid ? (unsigned long long)v : 0ull);
-      if ((threadIdx.x & 31) == 0 && mx) atomicMax(&s_max, mx);
+      count_group(g >= 0, g, s_cnt);
+      mx = (unsigned long long)v > mx ? (unsigned long long)v : mx;
     }
   }
   const long long tot = block_sum_ll(s, ws);
   if (threadIdx.x == 0) tile_sums[blockIdx.x] = tot;
   if (grouping) {
+    mx = warp_max_u64(mx);
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(&s_max, mx);
     __syncthreads();
-    if (threadIdx.x < kMaxGroups && s_rows[threadIdx.x]) {
-      atomicAdd(&acc->num_rows[threadIdx.x], s_rows[threadIdx.x]);
-      atomicAdd(&acc->num_nnzc[threadIdx.x], s_nzc[threadIdx.x]);
-      atomicAdd(&acc->num_nprod[threadIdx.x], s_np[threadIdx.x]);
-      atomicAdd(&acc->num_nnza[threadIdx.x], s_nza[threadIdx.x]);
-    }
-    if (threadIdx.x == 0) atomicMax(&acc->max_nnz, s_max);
+    if (threadIdx.x < kMaxGroups && s_cnt[threadIdx.x])
+      atomicAdd(&acc->num_rows[threadIdx.x], (unsigned long long)s_cnt[threadIdx.x]);
+    if (threadIdx.x == 0 && s_max) atomicMax(&acc->max_nnz, s_max);
+  }
+}
+
+// Per-group sums for spgemm_get_stats (n_prod, nnz(A), nnz(C) of each group's rows): run on
+// demand, off the SpGEMM critical path.
+__global__ __launch_bounds__(kSetupThreads) void k_group_stats(long long m, const uint8_t* __restrict__ grp1,
+                                                               const uint8_t* __restrict__ grp2,
+                                                               const int64_t* __restrict__ nprod,
+                                                               const int64_t* __restrict__ a_rpt,
+                                                               const int64_t* __restrict__ c_rpt, DevAcc* acc) {
+  __shared__ unsigned long long s[5][kMaxGroups];
+  for (int i = threadIdx.x; i < 5 * kMaxGroups; i += blockDim.x) (&s[0][0])[i] = 0;
+  __syncthreads();
+  const long long i = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
+  int g1 = -1, g2 = -1;
+  unsigned long long np = 0, na = 0, nc = 0;
+  if (i < m) {
+    g1 = grp1[i] == 0xFF ? -1 : grp1[i];
+    g2 = grp2[i] == 0xFF ? -1 : grp2[i];
+    np = (unsigned long long)nprod[i];
+    na = (unsigned long long)(a_rpt[i + 1] - a_rpt[i]);
+    nc = (unsigned long long)(c_rpt[i + 1] - c_rpt[i]);
+  }
+  {
+    const unsigned long long v[2] = {np, na};
+    unsigned long long* const d[2] = {s[0], s[1]};
+    warp_group_add<2>(g1 >= 0, g1, v, d);
+  }
+  {
+    const unsigned long long v[3] = {np, na, nc};
+    unsigned long long* const d[3] = {s[2], s[3], s[4]};
+    warp_group_add<3>(g2 >= 0, g2, v, d);
+  }
+  __syncthreads();
+  if (threadIdx.x < kMaxGroups) {
+    const int g = threadIdx.x;
+    if (s[0][g]) atomicAdd(&acc->sym_nprod[g], s[0][g]);
+    if (s[1][g]) atomicAdd(&acc->sym_nnza[g], s[1][g]);
+    if (s[2][g]) atomicAdd(&acc->num_nprod[g], s[2][g]);
+    if (s[3][g]) atomicAdd(&acc->num_nnza[g], s[3][g]);
+    if (s[4][g]) atomicAdd(&acc->num_nnzc[g], s[4][g]);
   }
 }
 
@@ -266,19 +365,26 @@ __global__ void k_splits(long long m, const int64_t* __restrict__ excl, int npar
 
 }  // namespace
 
-cudaError_t launch_nprod_group(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,
-                               const int64_t* b_rpt, int64_t* nprod, uint8_t* grp, int64_t* c_rpt,
-                               DevAcc* acc, Bounds b, int lpr_log2) {
+cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
+                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
+                               int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
+                               int* nlaunch) {
   if (m == 0) return cudaSuccess;
-  const int lpr = 1 << lpr_log2;
-  const long long rpb = kSetupThreads / lpr;
-  const unsigned grid = (unsigned)((m + rpb - 1) / rpb);
-  switch (lpr_log2) {
-#define SPG_CASE(L) case L: k_nprod_group<(1 << L)><<<grid, kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod, grp, c_rpt, acc, b); break;
-    SPG_CASE(0) SPG_CASE(1) SPG_CASE(2) SPG_CASE(3) SPG_CASE(4) SPG_CASE(5)
-#undef SPG_CASE
-    default: return cudaErrorInvalidValue;
+  if (bmm && k > 0) {
+    k_brow_minmax<<<(unsigned)((k + kSetupThreads - 1) / kSetupThreads), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm);
+    if (nlaunch) ++*nlaunch;
   }
+  const unsigned grid = (unsigned)((m + kSetupThreads - 1) / kSetupThreads);
+  k_nprod_group<<<grid, kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b);
+  if (nlaunch) ++*nlaunch;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1, const uint8_t* grp2,
+                               const int64_t* nprod, const int64_t* a_rpt, const int64_t* c_rpt, DevAcc* acc) {
+  if (m == 0) return cudaSuccess;
+  k_group_stats<<<(unsigned)((m + kSetupThreads - 1) / kSetupThreads), kSetupThreads, 0, s>>>(m, grp1, grp2, nprod,
+                                                                                             a_rpt, c_rpt, acc);
   return cudaGetLastError();
 }
 
@@ -294,12 +400,11 @@ size_t scan_workspace_bytes(long long m) {
   return (size_t)((m + kScanTile - 1) / kScanTile + 1) * sizeof(long long);
 }
 
-static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const int64_t* nprod,
-                                  const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
+static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, uint8_t* grp2, DevAcc* acc, Bounds b,
                                   long long* tile_ws, long long* total_out, int* nlaunch) {
   if (m == 0) return cudaSuccess;
   const long long ntiles = (m + kScanTile - 1) / kScanTile;
-  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, nprod, a_rpt, grp2, acc, b);
+  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, grp2, acc, b);
   k_scan_tiles<<<1, 1024, 0, s>>>(ntiles, tile_ws);
   k_scan_down<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, total_out);
   if (nlaunch) *nlaunch += 3;
@@ -309,7 +414,8 @@ static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const
 cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const int64_t* nprod,
                                   const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
                                   long long* tile_ws, int* nlaunch) {
-  return scan_inclusive(s, m, c_rpt + 1, nprod, a_rpt, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
+  (void)nprod; (void)a_rpt;
+  return scan_inclusive(s, m, c_rpt + 1, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
 }
 
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
@@ -327,7 +433,7 @@ cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, 
     const long long rpb = kSetupThreads / 32;
     k_nprod_only<<<(unsigned)((m + rpb - 1) / rpb), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod_scan + 1);
     Bounds none{};
-    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
+    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
     if (e != cudaSuccess) return e;
   }
   k_splits<<<(nparts + 1 + 255) / 256, 256, 0, s>>>(m, nprod_scan, nparts, splits_dev);

@@ -35,17 +35,56 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   int* table = smem + g * T;
   const long long ridx = (long long)blockIdx.x * RPB + g;
 
+  const bool active = ridx < a.nrows;
+  const int row = active ? a.rows[ridx] : -1;
+  // Range-offset hash: when the row's column span R fits 4*T bytes the table
+  // is a byte-flag array indexed by key - lo_i (collision-free; idempotent plain stores, no
+  // atomics, conflict-free for consecutive keys); the count is the number of set flags.
+  // Spans up to 32*T columns use a bitmap instead (red.shared.or; wider spans mean fewer
+  // same-word collisions inside a warp).
+  bool direct = false, bitmap = false;
+  int lo = 0, words = 0;
+  if (active && a.rlohi != nullptr) {
+    const int2 r = __ldg(a.rlohi + row);
+    const long long R = (long long)r.y - r.x + 1;
+    if (R > 0 && R <= 4LL * T) { direct = true; lo = r.x; words = (int)((R + 3) >> 2); }
+    else if (R > 0 && R <= 32LL * T) { direct = bitmap = true; lo = r.x; words = (int)((R + 31) >> 5); }
+  }
   int4* t4 = reinterpret_cast<int4*>(table);
+  if (direct) {
+    for (int s = t; s < (words + 3) / 4; s += TPR) t4[s] = make_int4(0, 0, 0, 0);
+  } else {
 #pragma unroll 4
-  for (int s = t; s < T / 4; s += TPR) t4[s] = make_int4(-1, -1, -1, -1);
+    for (int s = t; s < T / 4; s += TPR) t4[s] = make_int4(-1, -1, -1, -1);
+  }
   if (OPT && threadIdx.x == 0) { s_cnt = 0; s_abort = 0; }
+  if (threadIdx.x == 0) s_lcnt = 0;
   Grp<TPR>::sync();
 
   int cnt = 0;
-  const bool active = ridx < a.nrows;
-  const int row = active ? a.rows[ridx] : -1;
-  const SKeys K{smem_u32(table)};
+  const unsigned tb = smem_u32(table);
+  const SKeys K{tb};
   const int long_len = TPR > 32 ? a.long_len : 0;
+  if (direct) {  // uniform within the row group (CTA-uniform when TPR > 32)
+    auto f = [&](int key, int) {
+      const unsigned d = (unsigned)(key - lo);
+      if (bitmap) red_or_s(tb + 4u * (d >> 5), 1u << (d & 31));
+      else st_s8(tb + d, 1);
+    };
+    if (active)
+      for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
+                                          a.vw_log2, f, NoStop{}, long_len, &s_lcnt);
+    if constexpr (TPR > 32) {
+      if (long_len > 0)
+        for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
+                                             TPR, long_len, s_list, &s_lcnt, f, NoStop{});
+    }
+    Grp<TPR>::sync();
+    for (int w = t; w < words; w += TPR) cnt += __popc((unsigned)table[w]);  // 0/1 bytes or bits
+    const int tot = Grp<TPR>::sum32(cnt, reinterpret_cast<int*>(ws));
+    if (t == 0 && row >= 0) a.c_cnt[row] = tot;
+    return;
+  }
   if constexpr (OPT) {
     const unsigned ab = smem_u32(&s_abort);
     auto stop = [ab]() { return lds_s32(ab) != 0; };
@@ -56,7 +95,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
     };
     if (active)
       for_each_product<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
-                                         a.vw_log2, f, stop, long_len);
+                                         a.vw_log2, f, stop, long_len, &s_lcnt);
     if (long_len > 0)
       for_long_products<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
                                           TPR, long_len, s_list, &s_lcnt, f, stop);
@@ -68,7 +107,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
     };
     if (active)
       for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
-                                          a.vw_log2, f, NoStop{}, long_len);
+                                          a.vw_log2, f, NoStop{}, long_len, &s_lcnt);
     if constexpr (TPR > 32) {
       if (long_len > 0)
         for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
@@ -86,7 +125,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
       }
     }
   } else {
-    const long long tot = Grp<TPR>::sum(cnt, ws);
+    const int tot = Grp<TPR>::sum32(cnt, reinterpret_cast<int*>(ws));
     if (t == 0 && row >= 0) a.c_cnt[row] = tot;
   }
 }
@@ -109,6 +148,7 @@ __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
     if (T > a.slab_T) T = a.slab_T;
     int4* t4 = reinterpret_cast<int4*>(table);
     for (long long s = t; s < T / 4; s += 1024) t4[s] = make_int4(-1, -1, -1, -1);
+    if (t == 0) s_lcnt = 0;
     __syncthreads();
     int cnt = 0;
     const GKeys K{table};
@@ -118,7 +158,7 @@ __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
       cnt += ins;
     };
     for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, 1024,
-                                        a.vw_log2, f, NoStop{}, a.long_len);
+                                        a.vw_log2, f, NoStop{}, a.long_len, &s_lcnt);
     if (a.long_len > 0)
       for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
                                            a.long_len, s_list, &s_lcnt, f, NoStop{});

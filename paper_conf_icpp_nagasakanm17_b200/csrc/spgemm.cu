@@ -55,6 +55,7 @@ struct spgemm_ctx {
   cudaStream_t stream = nullptr;
   spgemm_allocator_t alloc{};
   bool user_alloc = false;
+  cudaMemPool_t pool = nullptr;  // private stream-ordered pool; memory retained across calls
   cudaStream_t gs[kNumStreams]{};
   cudaEvent_t fork_ev = nullptr;
   cudaEvent_t join_ev[kNumStreams]{};
@@ -64,6 +65,7 @@ struct spgemm_ctx {
   // options
   int sym_min_group = -1, num_min_group = -1, fill_limit = 0, use_streams = 1, validate = 0, lanes = 0;
   int long_len = 0;  // 0 auto, -1 off
+  int range_hash = 1;  // 1: range-offset hash where a row's column span fits
   int timing = 1;
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -74,8 +76,9 @@ struct spgemm_ctx {
   const int32_t *a_col = nullptr, *b_col = nullptr;
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
-  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, slab_sym;
+  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, slab_sym, bmm, rlohi;
   bool perm2_ready = false;
+  bool group_sums_done = false;  // per-group n_prod/nnz sums (computed on demand by get_stats)
   DevAcc* hacc = nullptr;      // pinned
   long long* hends = nullptr;  // pinned: a_rpt[0], a_rpt[m], b_rpt[0], b_rpt[k]
   DevAcc snap1{}, snap2{};
@@ -112,11 +115,11 @@ spgemm_status_t buf_alloc(spgemm_handle_t h, Buf& b, size_t bytes) {
     b.p = h->alloc.alloc(bytes, (void*)h->stream, h->alloc.ctx);
     if (!b.p) return fail(h, SPGEMM_ERR_OOM, "allocator returned NULL for " + std::to_string(bytes) + " bytes");
   } else {
-    cudaError_t e = cudaMallocAsync(&b.p, bytes, h->stream);
+    cudaError_t e = cudaMallocFromPoolAsync(&b.p, bytes, h->pool, h->stream);
     if (e != cudaSuccess) {
       cudaGetLastError();
       b.p = nullptr;
-      return fail(h, SPGEMM_ERR_OOM, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
+      return fail(h, SPGEMM_ERR_OOM, std::string("cudaMallocFromPoolAsync: ") + cudaGetErrorString(e));
     }
   }
   b.bytes = bytes;
@@ -135,7 +138,8 @@ void buf_free(spgemm_handle_t h, Buf& b) {
 }
 
 void release_state(spgemm_handle_t h) {
-  Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow, &h->slab_sym};
+  Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow, &h->slab_sym,
+                &h->bmm, &h->rlohi};
   for (Buf* b : all) buf_free(h, *b);
   h->state = 0;
   h->perm2_ready = false;
@@ -283,6 +287,20 @@ spgemm_status_t spgemm_create(spgemm_handle_t* out, int device, void* stream, co
       e = cudaEventCreate(&h->gstart[p][i]);
       if (e == cudaSuccess) e = cudaEventCreate(&h->gstop[p][i]);
     }
+  if (e == cudaSuccess && !h->user_alloc) {
+    // Private pool whose memory stays mapped between calls (release threshold = max): the
+    // default pool unmaps at every synchronisation, which re-maps the global-memory hash
+    // slabs (up to hundreds of MB) on every call.  Trimmed in spgemm_destroy.
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = device;
+    e = cudaMemPoolCreate(&h->pool, &props);
+    if (e == cudaSuccess) {
+      unsigned long long thr = ~0ull;
+      e = cudaMemPoolSetAttribute(h->pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
   if (e == cudaSuccess) e = cudaMallocHost(&h->hacc, sizeof(DevAcc));
   if (e == cudaSuccess) e = cudaMallocHost(&h->hends, 4 * sizeof(long long));
   *out = h;
@@ -311,6 +329,10 @@ spgemm_status_t spgemm_destroy(spgemm_handle_t h) {
       }
     if (h->hacc) cudaFreeHost(h->hacc);
     if (h->hends) cudaFreeHost(h->hends);
+    if (h->pool) {
+      cudaMemPoolTrimTo(h->pool, 0);
+      cudaMemPoolDestroy(h->pool);
+    }
   }
   delete h;
   return SPGEMM_OK;
@@ -337,6 +359,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       if (v <= 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "budget must be > 0");
       h->ws_budget = v; break;
     case SPGEMM_OPT_TIMING: h->timing = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANGE_HASH: h->range_hash = v ? 1 : 0; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -385,15 +408,23 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   ALLOC(h->perm1, sizeof(int32_t) * m);
   ALLOC(h->perm2, sizeof(int32_t) * m);
   ALLOC(h->tiles, scan_workspace_bytes(m));
+  if (h->range_hash) {
+    ALLOC(h->bmm, sizeof(int2) * std::max<int64_t>(k, 1));
+    ALLOC(h->rlohi, sizeof(int2) * m);
+  }
   if (h->timing) CK(cudaEventRecord(h->ev[0], h->stream));
   if (h->validate) {
     CK(launch_validate(h->stream, m, k, n, a_rpt, a_col, b_rpt, b_col, &dacc->err_flags));
     ++launches;
   }
-  // (1)+(2): n_prod per row (Alg. 2) and group ids / histogram
-  CK(launch_nprod_group(h->stream, m, a_rpt, a_col, b_rpt, static_cast<int64_t*>(h->nprod.p),
-                        static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h->sym_min_group), 3));
-  ++launches;
+  // (1)+(2): n_prod per row (Alg. 2), column spans, group ids / histogram
+  {
+    int nl = 0;
+    CK(launch_nprod_group(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, static_cast<int2*>(h->bmm.p),
+                          static_cast<int64_t*>(h->nprod.p), static_cast<int2*>(h->rlohi.p),
+                          static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h->sym_min_group), &nl));
+    launches += nl;
+  }
   CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
   CK(cudaMemcpyAsync(h->hends + 0, a_rpt, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
   CK(cudaMemcpyAsync(h->hends + 1, a_rpt + m, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
@@ -431,6 +462,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.c_cnt = c_rpt + 1;
   sa.vw_log2 = h->vw_log2;
   sa.long_len = long_len_of(h);
+  sa.rlohi = static_cast<const int2*>(h->rlohi.p);
   sa.overflow_rows = static_cast<int32_t*>(h->overflow.p);
   sa.overflow_count = &dacc->overflow_count;
   const int T_opt = kSymGroups[kSymOptimistic].T, BS_opt = kSymGroups[kSymOptimistic].BS;
@@ -501,13 +533,9 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   st.max_row_nnz = (int64_t)h->snap2.max_nnz;
   for (int g = 0; g < kMaxGroups; ++g) {
     st.sym_rows[g] = (int64_t)h->snap1.sym_rows[g];
-    st.sym_nprod[g] = (int64_t)h->snap1.sym_nprod[g];
-    st.sym_nnza[g] = (int64_t)h->snap1.sym_nnza[g];
     st.num_rows[g] = (int64_t)h->snap2.num_rows[g];
-    st.num_nprod[g] = (int64_t)h->snap2.num_nprod[g];
-    st.num_nnza[g] = (int64_t)h->snap2.num_nnza[g];
-    st.num_nnzc[g] = (int64_t)h->snap2.num_nnzc[g];
   }
+  h->group_sums_done = false;
   st.sym_overflow_rows = h->snap2.overflow_count;
   st.kernel_launches_symbolic = launches;
   h->state = 1;
@@ -551,6 +579,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.c_rpt = h->c_rpt; na.c_col = c_col; na.c_val = c_val;
     na.vw_log2 = h->vw_log2;
     na.long_len = long_len_of(h);
+    na.rlohi = static_cast<const int2*>(h->rlohi.p);
     na.err_flags = &dacc->err_flags;
     Buf slab;
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
@@ -616,6 +645,30 @@ spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t* out) {
         *out = st;
         return fail(h, SPGEMM_ERR_INVALID_INPUT, "numeric row count disagreed with symbolic count");
       }
+    }
+  }
+  if (h->state == 1 && h->m > 0) {
+    if (!h->group_sums_done) {  // off the critical path: one extra kernel + copy, on demand
+      DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+      CK(launch_group_stats(h->stream, h->m, static_cast<uint8_t*>(h->grp1.p), static_cast<uint8_t*>(h->grp2.p),
+                            static_cast<int64_t*>(h->nprod.p), h->a_rpt, h->c_rpt, dacc));
+      CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
+      CK(cudaStreamSynchronize(h->stream));
+      for (int g = 0; g < kMaxGroups; ++g) {
+        h->stats.sym_nprod[g] = (int64_t)h->hacc->sym_nprod[g];
+        h->stats.sym_nnza[g] = (int64_t)h->hacc->sym_nnza[g];
+        h->stats.num_nprod[g] = (int64_t)h->hacc->num_nprod[g];
+        h->stats.num_nnza[g] = (int64_t)h->hacc->num_nnza[g];
+        h->stats.num_nnzc[g] = (int64_t)h->hacc->num_nnzc[g];
+      }
+      h->group_sums_done = true;
+    }
+    for (int g = 0; g < kMaxGroups; ++g) {
+      st.sym_nprod[g] = h->stats.sym_nprod[g];
+      st.sym_nnza[g] = h->stats.sym_nnza[g];
+      st.num_nprod[g] = h->stats.num_nprod[g];
+      st.num_nnza[g] = h->stats.num_nnza[g];
+      st.num_nnzc[g] = h->stats.num_nnzc[g];
     }
   }
   st.workspace_bytes = h->ws_cur;

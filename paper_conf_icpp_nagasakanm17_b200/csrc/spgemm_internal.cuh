@@ -38,10 +38,12 @@ struct GroupSpec {
 // rows above the last bound ("using the maximum hash table size for shared
 // memory"); rows that find more than the fill limit of distinct keys are retried in global
 // memory (group kSymGlobal).
+// Threads per row target ~8-16 products per thread at the group's bound (per-warp fixed costs
+// dominate below that).
 constexpr GroupSpec kSymGroups[] = {
     {16, 32, 4, 256},        {32, 64, 8, 256},         {128, 256, 16, 256},
-    {256, 512, 32, 256},     {512, 1024, 64, 64},      {1024, 2048, 128, 128},
-    {2048, 4096, 256, 256},  {4096, 8192, 512, 512},   {8192, 16384, 1024, 1024},
+    {256, 512, 32, 256},     {512, 1024, 32, 256},     {1024, 2048, 64, 64},
+    {2048, 4096, 128, 128},  {4096, 8192, 256, 256},   {8192, 16384, 512, 512},
     {16384, 32768, 1024, 1024},
     {-1, 32768, 1024, 1024},  // optimistic (no upper bound)
 };
@@ -62,8 +64,8 @@ constexpr int kNumGlobal = 10;
 constexpr int kNumNumGroups = 11;
 
 // Numeric per-row shared-memory layout: vals[T] | keys[T] | bucket[NB+1] | sidx[upper] ,
-// NB = T/2 (T/4 for the two largest tables) buckets for the bucket-rank sort.
-__host__ __device__ constexpr int num_nbuckets(int T) { return T <= 8192 ? T / 2 : T / 4; }
+// NB = T/2 (T/8 for the largest table) buckets for the bucket-rank sort.
+__host__ __device__ constexpr int num_nbuckets(int T) { return T <= 8192 ? T / 2 : T / 8; }
 __host__ __device__ constexpr int align16(int x) { return (x + 15) & ~15; }
 template <typename VT>
 __host__ __device__ constexpr int num_row_bytes(int T, long long upper) {
@@ -117,6 +119,8 @@ __device__ __forceinline__ int cas_s32(unsigned a, int cmp, int val) {
   asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(a), "r"(cmp), "r"(val));
   return old;
 }
+__device__ __forceinline__ void st_s8(unsigned a, int v) { asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v)); }
+__device__ __forceinline__ void red_or_s(unsigned a, unsigned v) { asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v)); }
 __device__ __forceinline__ void red_add_s(unsigned a, float v) { asm volatile("red.shared.add.f32 [%0], %1;" ::"r"(a), "f"(v)); }
 __device__ __forceinline__ void red_add_s(unsigned a, double v) { asm volatile("red.shared.add.f64 [%0], %1;" ::"r"(a), "d"(v)); }
 
@@ -128,7 +132,10 @@ struct SKeys {
 };
 struct GKeys {
   int* p;
-  __device__ __forceinline__ int ld(unsigned h) const { return ld_volatile(p + h); }
+  // ld.global.cg (L2, not L1-cached, not volatile): a slot changes only once (-1 -> key), so a
+  // stale -1 merely makes the following CAS report the real key; probes of independent
+  // products may overlap.
+  __device__ __forceinline__ int ld(unsigned h) const { return __ldcg(p + h); }
   __device__ __forceinline__ int cas(unsigned h, int c, int v) const { return atomicCAS(p + h, c, v); }
 };
 template <typename VT>
@@ -174,7 +181,7 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
                                                  const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                  const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
                                                  int row, int t, int tpr, int vwl, F&& f, S&& stop,
-                                                 int long_len = 0) {
+                                                 int long_len = 0, int* deferred = nullptr) {
   const long long a0 = __ldg(a_rpt + row);
   const int na = (int)(__ldg(a_rpt + row + 1) - a0);  // row-relative 32-bit indexing
   const int32_t* __restrict__ ac = opaque(a_col + a0);
@@ -200,7 +207,10 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
     if (jnn < na) { kknn = __ldg(ac + jnn); if (NUM) avnn = __ldg(avp + jnn); }
     const int32_t* __restrict__ bc = opaque(b_col + b0);
     const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
-    if (long_len > 0 && len > long_len) len = 0;  // deferred to for_long_products
+    if (long_len > 0 && len > long_len) {  // deferred to for_long_products
+      len = 0;
+      if (deferred) *deferred = 1;
+    }
 #pragma unroll 1
     for (int q = lane; q < len; q += 2 * vw) {
       const int k0 = __ldg(bc + q);
@@ -227,7 +237,9 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
 // Second pass (CTA-wide, every thread of the CTA must call it): the A row is rescanned in
 // chunks of kLongChunk entries; entries whose B row is longer than long_len go to a shared
 // list, and all tpr threads stride each listed B row (unrolled by 2).  s_list: kLongChunk
-// ints, s_cnt: one int, both shared.  A stopped (CHECK_STOP) thread keeps hitting barriers.
+// ints, s_cnt: one int, both shared; s_cnt must be 0 before pass 1 and is set by pass 1 when
+// it defers a row (otherwise this pass returns at once).  A stopped (CHECK_STOP) thread keeps
+// hitting barriers.
 constexpr int kLongChunk = 256;
 template <bool NUM, bool CHECK_STOP, typename VT, typename F, typename S>
 __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
@@ -236,8 +248,11 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
                                                   bool active, int row, int t, int tpr, int long_len, int* s_list,
                                                   int* s_cnt, F&& f, S&& stop) {
   const long long a0 = active ? __ldg(a_rpt + row) : 0;
-  const int na = active ? (int)(__ldg(a_rpt + row + 1) - a0) : 0;
   const int32_t* __restrict__ ac = a_col + a0;
+  __syncthreads();  // s_cnt doubles as the "some sub-group deferred a row" flag of pass 1
+  if (*(volatile int*)s_cnt == 0) return;  // CTA-uniform
+  const int na = active ? (int)(__ldg(a_rpt + row + 1) - a0) : 0;
+  __syncthreads();
   if (t == 0) *s_cnt = 0;
   __syncthreads();
   for (int c = 0; c < na; c += kLongChunk) {  // na is CTA-uniform
@@ -388,6 +403,24 @@ struct Grp {
     }
   }
 
+  // 32-bit group sum (REDUX on full warps); the result is valid on every thread of the group.
+  static __device__ __forceinline__ int sum32(int v, int* ws32) {
+    if constexpr (TPR < 32) {
+#pragma unroll
+      for (int o = TPR / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask(), v, o, TPR);
+      return v;
+    } else if constexpr (TPR == 32) {
+      return __reduce_add_sync(0xffffffffu, v);
+    } else {
+      const int w = __reduce_add_sync(0xffffffffu, v);
+      if (threadIdx.x == 0) *ws32 = 0;
+      __syncthreads();
+      if ((threadIdx.x & 31) == 0) atomicAdd(ws32, w);
+      __syncthreads();
+      return *ws32;
+    }
+  }
+
   static __device__ __forceinline__ long long sum(long long v, long long* ws) {
     long long t;
     excl_scan(v, &t, ws);
@@ -404,6 +437,7 @@ struct SymArgs {
   int64_t* c_cnt;          // c_rpt + 1: per-row nnz written here (scanned later)
   int vw_log2;             // lanes per B row = 1 << vw_log2 (Alg. 3/4 generalised)
   int long_len;            // CTA-per-row groups: B rows longer than this are walked by the CTA
+  const int2* rlohi;       // column span [lo_i, hi_i] of each row of C, or null (paper hash only)
   // optimistic group
   int32_t* overflow_rows; int* overflow_count; int fill_limit;
   // global fallback
@@ -418,14 +452,18 @@ struct NumArgs {
   const int64_t* c_rpt; int32_t* c_col; void* c_val;
   int vw_log2;
   int long_len;
+  const int2* rlohi;       // column span of each row of C, or null (paper hash only)
   int* err_flags;
   // global fallback
   void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;
 };
 
-cudaError_t launch_nprod_group(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,
-                               const int64_t* b_rpt, int64_t* nprod, uint8_t* grp, int64_t* c_rpt,
-                               DevAcc* acc, Bounds b, int lpr_log2);
+cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
+                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
+                               int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
+                               int* nlaunch);
+cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1, const uint8_t* grp2,
+                               const int64_t* nprod, const int64_t* a_rpt, const int64_t* c_rpt, DevAcc* acc);
 cudaError_t launch_group_scatter(cudaStream_t s, long long m, const uint8_t* grp, Offsets off,
                                  int* cursor, int32_t* perm);
 cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const int64_t* nprod,

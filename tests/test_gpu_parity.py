@@ -120,26 +120,39 @@ def _mixed_small():
     return A.with_values("uniform", 4)
 
 
+def _banded_small():
+    return synth.banded(20000, 2, 90, 60, seed=5, name="banded_small").with_values("uniform", 6)
+
+
+@pytest.mark.parametrize("range_hash", [0, 1])
 @pytest.mark.parametrize("group", list(range(0, 12)))
-def test_forced_symbolic_group(spg, group):
-    A = _mixed_small()
-    ref = oracle.spgemm(A, A, np.float64)
-    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": group})
-    assert_parity(got, ref, np.float64, what=f"sym group>={group}")
+def test_forced_symbolic_group(spg, group, range_hash):
+    for A in (_mixed_small(), _banded_small()):
+        ref = oracle.spgemm(A, A, np.float64)
+        got = run_gpu(spg, A, A, np.float64, {"sym_min_group": group, "range_hash": range_hash})
+        assert_parity(got, ref, np.float64, what=f"{A.name} sym group>={group} range_hash={range_hash}")
 
 
+@pytest.mark.parametrize("range_hash", [0, 1])
 @pytest.mark.parametrize("group", list(range(0, 11)))
-def test_forced_numeric_group(spg, group):
-    A = _mixed_small()
-    ref = oracle.spgemm(A, A, np.float32)
-    got = run_gpu(spg, A, A, np.float32, {"num_min_group": group})
-    assert_parity(got, ref, np.float32, what=f"num group>={group}")
+def test_forced_numeric_group(spg, group, range_hash):
+    for A in (_mixed_small(), _banded_small()):
+        ref = oracle.spgemm(A, A, np.float32)
+        got = run_gpu(spg, A, A, np.float32, {"num_min_group": group, "range_hash": range_hash})
+        assert_parity(got, ref, np.float32, what=f"{A.name} num group>={group} range_hash={range_hash}")
+
+
+@pytest.mark.parametrize("config", ["cant", "webbase", "mixed:protein", "mixed:economics"])
+def test_paper_hash_only(spg, config):
+    """The paper's multiplicative hash everywhere (range-offset hash disabled)."""
+    A = synth.config(config, "int")
+    check(spg, A, A, np.float32, exact=True, opts={"range_hash": 0}, what=f"{config} paper hash")
 
 
 def test_overflow_retry_in_global_memory(spg):
     A = _mixed_small()
     ref = oracle.spgemm(A, A, np.float64)
-    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16})
+    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16, "range_hash": 0})
     assert got[3]["sym_overflow_rows"] > 0
     assert_parity(got, ref, np.float64, what="overflow")
 
@@ -158,7 +171,8 @@ def test_long_row_cta_pass(spg, long_row, dtype):
     """B rows longer than long_row are walked by the whole CTA (second pass); 1 = every row."""
     A = _mixed_small()
     ref = oracle.spgemm(A.astype(dtype), A.astype(dtype), dtype)
-    for opts in ({"long_row": long_row}, {"long_row": long_row, "sym_min_group": 10, "sym_fill_limit": 64},
+    for opts in ({"long_row": long_row}, {"long_row": long_row, "range_hash": 0},
+                 {"long_row": long_row, "sym_min_group": 10, "sym_fill_limit": 64, "range_hash": 0},
                  {"long_row": long_row, "sym_min_group": 11, "num_min_group": 10}):
         got = run_gpu(spg, A, A, dtype, opts)
         assert_parity(got, ref, dtype, what=f"{opts}")
