@@ -61,6 +61,71 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
       const long long R = (long long)rr.y - rr.x + 1;
       if (R > 0 && R <= (long long)T) {  // uniform within the row group
         const int lo = rr.x;
+        const int long_len = TPR > 32 ? a.long_len : 0;
+        const int vwl = a.vw_log2;
+        const int ncopy = TPR >> vwl;  // one private accumulator row per sub-group
+        const long long Rp = (R + 3) & ~3LL;
+        const unsigned kb = smem_u32(Kp);
+        const bool priv = a.priv_ok &&
+                          ncopy * Rp * (long long)sizeof(VT) + Rp <= (long long)T * (long long)(sizeof(VT) + 4);
+        long long n_total;
+        const long long c0 = a.c_rpt[row];
+        const long long cn = a.c_rpt[row + 1] - c0;
+        VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+        int32_t* __restrict__ cc = a.c_col + c0;
+        if (priv) {
+          // Private accumulators: sub-group g adds into P[g][0..R) with plain read-modify-
+          // writes (its lanes hold distinct columns of one B row; WSYNC reconverges it per A
+          // non-zero), flags in the Rp bytes after the copies; the copies are summed in fixed
+          // order at compaction time, so values are deterministic run to run.
+          VT* P = Vp;
+          unsigned char* fl = reinterpret_cast<unsigned char*>(P + ncopy * Rp);
+          const unsigned fb = smem_u32(fl);
+          using V16 = typename Vec16<VT>::T;
+          constexpr int per = 16 / sizeof(VT);
+          V16* v16 = reinterpret_cast<V16*>(P);
+          for (long long s = t; s < ncopy * Rp / per; s += TPR) v16[s] = Vec16<VT>::zero();
+          int4* f4 = reinterpret_cast<int4*>(fl);
+          for (long long s = t; s < (Rp + 15) / 16; s += TPR) f4[s] = make_int4(0, 0, 0, 0);
+          Grp<TPR>::sync();
+          VT* __restrict__ mine = P + (t >> vwl) * Rp;
+          auto f = [&](int key, VT prod) {
+            const unsigned d = (unsigned)(key - lo);
+            st_s8(fb + d, 1);
+            mine[d] += prod;
+          };
+          for_each_product<true, false, VT, true>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
+                                                  a.b_col, static_cast<const VT*>(a.b_val), row, t, TPR, vwl, f,
+                                                  NoStop{}, long_len, s_lcnt);
+          if constexpr (TPR > 32) {
+            if (long_len > 0)
+              for_long_products<true, false, VT, true>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
+                                                       a.b_col, static_cast<const VT*>(a.b_val), true, row, t, TPR,
+                                                       long_len, s_list, s_lcnt, f, NoStop{});
+          }
+          Grp<TPR>::sync();
+          const int words = (int)(Rp >> 2);
+          const int pw = (words + TPR - 1) / TPR;
+          const int w0 = t * pw, w1 = min(words, w0 + pw);
+          const unsigned* fw = reinterpret_cast<const unsigned*>(fl);
+          long long loc = 0;
+          for (int w = w0; w < w1; ++w) loc += __popc(fw[w]);
+          long long r = Grp<TPR>::excl_scan(loc, &n_total, ws);
+          if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
+          for (int w = w0; w < w1; ++w) {
+            unsigned bits = fw[w];
+            while (bits) {
+              const int d = w * 4 + ((__ffs(bits) - 1) >> 3);
+              bits &= bits - 1;
+              VT v = P[d];
+              for (int c = 1; c < ncopy; ++c) v += P[c * Rp + d];
+              if (r < cn) { cc[r] = lo + d; cv[r] = v; }
+              ++r;
+            }
+          }
+          Grp<TPR>::sync();
+          return;
+        }
         const int words = (int)((R + 3) >> 2);  // 4 flag bytes per word
         using V16 = typename Vec16<VT>::T;
         constexpr int per = 16 / sizeof(VT);
@@ -69,13 +134,11 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
         int4* k4 = reinterpret_cast<int4*>(Kp);
         for (int s = t; s < (words + 3) / 4; s += TPR) k4[s] = make_int4(0, 0, 0, 0);
         Grp<TPR>::sync();
-        const unsigned kb = smem_u32(Kp);
         auto f = [&](int key, VT prod) {
           const unsigned d = (unsigned)(key - lo);
           st_s8(kb + d, 1);
           V.add(d, prod);
         };
-        const int long_len = TPR > 32 ? a.long_len : 0;
         for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
                                           static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
                                           long_len, s_lcnt);
@@ -91,13 +154,8 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
         const int w0 = t * pw, w1 = min(words, w0 + pw);
         long long loc = 0;
         for (int w = w0; w < w1; ++w) loc += __popc((unsigned)Kp[w]);
-        long long n_total;
         long long r = Grp<TPR>::excl_scan(loc, &n_total, ws);
-        const long long c0 = a.c_rpt[row];
-        const long long cn = a.c_rpt[row + 1] - c0;
         if (t == 0 && cn != n_total) atomicOr(a.err_flags, 2);
-        VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
-        int32_t* __restrict__ cc = a.c_col + c0;
         for (int w = w0; w < w1; ++w) {
           unsigned bits = (unsigned)Kp[w];
           while (bits) {
@@ -387,7 +445,7 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : 0;
   num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
-                   s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr);
+                          s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr);
 }
 
 template <typename VT>

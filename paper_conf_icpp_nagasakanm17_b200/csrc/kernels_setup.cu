@@ -37,36 +37,45 @@ __device__ __forceinline__ void count_group(bool valid, int g, int* s_cnt) {
 constexpr int kLongA = 16;
 __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, const int64_t* __restrict__ b_rpt,
                                                                const int32_t* __restrict__ b_col,
-                                                               int2* __restrict__ bmm) {
+                                                               int2* __restrict__ bmm, int* __restrict__ unsorted) {
   const int lane = threadIdx.x & 31;
   const long long row = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
   long long b0 = 0, b1 = 0;
   if (row < k) { b0 = b_rpt[row]; b1 = b_rpt[row + 1]; }
   const bool is_long = b1 - b0 > kLongA;
   int mn = INT_MAX, mx = -1;
-  if (!is_long)
+  bool bad = false;  // some B row is not strictly increasing (duplicates or unsorted)
+  if (!is_long) {
+    int prev = -1;
     for (long long j = b0; j < b1; ++j) {
       const int c = __ldg(b_col + j);
       mn = min(mn, c); mx = max(mx, c);
+      bad |= c <= prev;
+      prev = c;
     }
+  }
   unsigned longs = __ballot_sync(0xffffffffu, is_long);
   while (longs) {
     const int src = __ffs(longs) - 1;
     longs &= longs - 1;
     const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
     int pmn = INT_MAX, pmx = -1;
+    bool pbad = false;
     for (long long j = s0 + lane; j < s1; j += 32) {
       const int c = __ldg(b_col + j);
       pmn = min(pmn, c); pmx = max(pmx, c);
+      if (j > s0) pbad |= c <= __ldg(b_col + j - 1);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
       pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
       pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
     }
+    bad |= __any_sync(0xffffffffu, pbad) && lane == src;
     if (lane == src) { mn = pmn; mx = pmx; }
   }
   if (row < k) bmm[row] = make_int2(mn, mx);
+  if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(unsorted, 1);
 }
 
 // One row per thread; rows longer than kLongA entries are summed by the whole warp
@@ -371,7 +380,8 @@ cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const i
                                int* nlaunch) {
   if (m == 0) return cudaSuccess;
   if (bmm && k > 0) {
-    k_brow_minmax<<<(unsigned)((k + kSetupThreads - 1) / kSetupThreads), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm);
+    k_brow_minmax<<<(unsigned)((k + kSetupThreads - 1) / kSetupThreads), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm,
+                                                                                               &acc->b_unsorted);
     if (nlaunch) ++*nlaunch;
   }
   const unsigned grid = (unsigned)((m + kSetupThreads - 1) / kSetupThreads);

@@ -23,20 +23,10 @@ struct NoStop {
   __device__ __forceinline__ bool operator()() const { return false; }
 };
 
-template <int T, int TPR, int BS, bool OPT>
-__global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
-  extern __shared__ __align__(16) int smem[];
-  __shared__ long long ws[33];
-  __shared__ int s_cnt, s_abort, s_lcnt;
-  __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
-  constexpr int RPB = BS / TPR;
-  static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
-  const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
-  int* table = smem + g * T;
-  const long long ridx = (long long)blockIdx.x * RPB + g;
-
-  const bool active = ridx < a.nrows;
-  const int row = active ? a.rows[ridx] : -1;
+// One row (all TPR threads of its row group call it; the table is the group's slice).
+template <int T, int TPR, bool OPT>
+__device__ __forceinline__ void sym_row(const SymArgs& a, bool active, int row, int t, int* table, long long* ws,
+                                        int& s_cnt, int& s_abort, int& s_lcnt, int* s_list) {
   // Range-offset hash: when the row's column span R fits 4*T bytes the table
   // is a byte-flag array indexed by key - lo_i (collision-free; idempotent plain stores, no
   // atomics, conflict-free for consecutive keys); the count is the number of set flags.
@@ -128,6 +118,22 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
     const int tot = Grp<TPR>::sum32(cnt, reinterpret_cast<int*>(ws));
     if (t == 0 && row >= 0) a.c_cnt[row] = tot;
   }
+}
+
+template <int T, int TPR, int BS, bool OPT>
+__global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
+  extern __shared__ __align__(16) int smem[];
+  __shared__ long long ws[33];
+  __shared__ int s_cnt, s_abort, s_lcnt;
+  __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
+  constexpr int RPB = BS / TPR;
+  static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
+  const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
+  int* table = smem + g * T;
+  const long long ridx = (long long)blockIdx.x * RPB + g;
+  const bool active = ridx < a.nrows;
+  const int row = active ? a.rows[ridx] : -1;
+  sym_row<T, TPR, OPT>(a, active, row, t, table, ws, s_cnt, s_abort, s_lcnt, s_list);
 }
 
 // Global-memory table per CTA (slab of slab_T ints), one row at a time; table size

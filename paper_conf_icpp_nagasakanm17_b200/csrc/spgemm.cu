@@ -580,6 +580,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.vw_log2 = h->vw_log2;
     na.long_len = long_len_of(h);
     na.rlohi = static_cast<const int2*>(h->rlohi.p);
+    na.priv_ok = h->snap1.b_unsorted ? 0 : 1;
     na.err_flags = &dacc->err_flags;
     Buf slab;
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];

@@ -83,6 +83,7 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   long long nnzc;
   int overflow_count;
   int err_flags;  // bit0 invalid input, bit1 numeric row count mismatch
+  int b_unsorted;  // some B row is not strictly increasing (disables private accumulators)
   int cursor[2][kMaxGroups];
 };
 
@@ -176,7 +177,7 @@ __device__ __forceinline__ unsigned probe(const Keys& K, unsigned mask, int key,
 // Load balance (CTA-per-row groups): with long_len > 0 a sub-group skips B rows longer than
 // long_len; the caller then runs for_long_products, where the whole CTA walks each of them
 // (hub columns of power-law graphs would otherwise serialise a CTA behind one sub-group).
-template <bool NUM, bool CHECK_STOP, typename VT, typename F, typename S>
+template <bool NUM, bool CHECK_STOP, typename VT, bool WSYNC = false, typename F, typename S>
 __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
                                                  const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                  const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
@@ -187,50 +188,67 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
   const int32_t* __restrict__ ac = opaque(a_col + a0);
   const VT* __restrict__ avp = NUM ? opaque(a_val + a0) : nullptr;
   const int vw = 1 << vwl, sub = t >> vwl, lane = t & (vw - 1), nsub = tpr >> vwl;
-  int j = sub;
-  if (j >= na) return;
-  int kk = __ldg(ac + j);
-  VT av = NUM ? __ldg(avp + j) : VT(0);
-  int jn = j + nsub;
-  int kkn = 0;
-  VT avn = VT(0);
-  if (jn < na) { kkn = __ldg(ac + jn); if (NUM) avn = __ldg(avp + jn); }
-  long long b0 = __ldg(b_rpt + kk);
-  int len = (int)(__ldg(b_rpt + kk + 1) - b0);
-  while (true) {
+  // WSYNC: reconverge the sub-group after every A non-zero (callers that update per-sub-group
+  // private accumulators with plain read-modify-writes rely on it)
+  const unsigned sg = vw >= 32 ? 0xffffffffu : (((1u << vw) - 1u) << ((threadIdx.x & 31) & ~(vw - 1)));
+  // Sub-group `sub` owns A non-zeros sub, sub + nsub, sub + 2*nsub, ... (Alg. 4's warp-per-a_ik,
+  // interleaved); they are taken in batches of vw: lane l fetches the metadata of the l-th
+  // non-zero of the batch (col_A, val_A, rpt_B pair — vw independent gathers in flight, the next
+  // batch prefetched), then the sub-group walks the batch with shuffle broadcasts.
+  const int stride = nsub * vw;
+  int jb = sub + nsub * lane;  // this lane's non-zero in the current batch
+  if (sub >= na) return;
+  int kk = 0, len = 0;
+  long long b0 = 0;
+  VT av = VT(0);
+  if (jb < na) {
+    kk = __ldg(ac + jb);
+    if (NUM) av = __ldg(avp + jb);
+    b0 = __ldg(b_rpt + kk);
+    len = (int)(__ldg(b_rpt + kk + 1) - b0);
+  }
+  for (int base = sub; base < na; base += stride) {
+    const int cnt = min(vw, (na - base + nsub - 1) / nsub);  // sub-group-uniform
+    // prefetch the next batch
+    const int jn = jb + stride;
+    int kkn = 0, lenn = 0;
     long long b0n = 0;
-    int lenn = 0;
-    if (jn < na) { b0n = __ldg(b_rpt + kkn); lenn = (int)(__ldg(b_rpt + kkn + 1) - b0n); }
-    const int jnn = jn + nsub;
-    int kknn = 0;
-    VT avnn = VT(0);
-    if (jnn < na) { kknn = __ldg(ac + jnn); if (NUM) avnn = __ldg(avp + jnn); }
-    const int32_t* __restrict__ bc = opaque(b_col + b0);
-    const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
-    if (long_len > 0 && len > long_len) {  // deferred to for_long_products
-      len = 0;
-      if (deferred) *deferred = 1;
+    VT avn = VT(0);
+    if (jn < na) {
+      kkn = __ldg(ac + jn);
+      if (NUM) avn = __ldg(avp + jn);
+      b0n = __ldg(b_rpt + kkn);
+      lenn = (int)(__ldg(b_rpt + kkn + 1) - b0n);
     }
+    for (int e = 0; e < cnt; ++e) {
+      const long long eb0 = __shfl_sync(sg, b0, e, vw);
+      int elen = __shfl_sync(sg, len, e, vw);
+      const VT eav = NUM ? __shfl_sync(sg, av, e, vw) : VT(0);
+      if (long_len > 0 && elen > long_len) {  // deferred to for_long_products
+        elen = 0;
+        if (deferred) *deferred = 1;
+      }
+      const int32_t* __restrict__ bc = opaque(b_col + eb0);
+      const VT* __restrict__ bv = NUM ? opaque(b_val + eb0) : nullptr;
 #pragma unroll 1
-    for (int q = lane; q < len; q += 2 * vw) {
-      const int k0 = __ldg(bc + q);
-      const VT v0 = NUM ? __ldg(bv + q) : VT(0);
-      const bool h1 = q + vw < len;
-      int k1 = 0;
-      VT v1 = VT(0);
-      if (h1) { k1 = __ldg(bc + q + vw); if (NUM) v1 = __ldg(bv + q + vw); }
-      if (CHECK_STOP && stop()) return;
-      f(k0, av * v0);
-      if (h1) {
-        if (CHECK_STOP && stop()) return;
-        f(k1, av * v1);
+      for (int q = lane; q < elen; q += 2 * vw) {
+        const int k0 = __ldg(bc + q);
+        const VT v0 = NUM ? __ldg(bv + q) : VT(0);
+        const bool h1 = q + vw < elen;
+        int k1 = 0;
+        VT v1 = VT(0);
+        if (h1) { k1 = __ldg(bc + q + vw); if (NUM) v1 = __ldg(bv + q + vw); }
+        // CHECK_STOP: a stopped lane skips its products (at most one insert after the flag is
+        // raised); the sub-group leaves together at the next entry boundary.
+        if (!(CHECK_STOP && stop())) f(k0, eav * v0);
+        if (h1 && !(CHECK_STOP && stop())) f(k1, eav * v1);
+      }
+      if constexpr (WSYNC || CHECK_STOP) __syncwarp(sg);
+      if constexpr (CHECK_STOP) {
+        if (__any_sync(sg, stop())) return;
       }
     }
-    if (jn >= na) return;
-    if (CHECK_STOP && stop()) return;
-    j = jn;
-    kk = kkn; av = avn; b0 = b0n; len = lenn;
-    jn = jnn; kkn = kknn; avn = avnn;
+    jb = jn; kk = kkn; av = avn; b0 = b0n; len = lenn;
   }
 }
 
@@ -241,7 +259,7 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
 // it defers a row (otherwise this pass returns at once).  A stopped (CHECK_STOP) thread keeps
 // hitting barriers.
 constexpr int kLongChunk = 256;
-template <bool NUM, bool CHECK_STOP, typename VT, typename F, typename S>
+template <bool NUM, bool CHECK_STOP, typename VT, bool WSYNC = false, typename F, typename S>
 __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
                                                   const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                   const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
@@ -286,6 +304,7 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
           f(k1, av * v1);
         }
       }
+      if constexpr (WSYNC) __syncwarp();
     }
     __syncthreads();
     if (t == 0) *s_cnt = 0;
@@ -453,6 +472,7 @@ struct NumArgs {
   int vw_log2;
   int long_len;
   const int2* rlohi;       // column span of each row of C, or null (paper hash only)
+  int priv_ok;             // B rows strictly increasing: private per-sub-group accumulators allowed
   int* err_flags;
   // global fallback
   void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;

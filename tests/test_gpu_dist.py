@@ -1,0 +1,64 @@
+"""Row-partitioned C = A^2 through the product callables (spgemm_row_partition and the CUDA
+two-phase SpGEMM) with two ranks sharing cuda:0 over gloo (NCCL needs one GPU per rank; the
+box has one) — -m gpu.  Concatenated shards must equal the oracle bit-exactly (int values)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, name, out_dir):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import synth
+        import paper_conf_icpp_nagasakanm17_b200 as P
+        from paper_conf_icpp_nagasakanm17_b200.dist import (cuda_local_multiply, cuda_partition,
+                                                            distributed_spgemm)
+        torch.cuda.set_device(0)
+        A = None
+        if rank == 0:
+            A = P.CsrMatrix.from_host(synth.config(name, "int"), "cuda:0", torch.float32)
+        with P.Handle(0) as h:
+            res, grpt = distributed_spgemm(A, None, device="cuda:0", dtype=torch.float32, square=True,
+                                           partition=cuda_partition(h), local_multiply=cuda_local_multiply(h),
+                                           gather_rpt=True)
+            torch.cuda.synchronize()
+            rpt, col, val = res.C.numpy()
+        np.savez(os.path.join(out_dir, f"r{rank}.npz"), col=col, val=val, splits=np.array(res.splits),
+                 grpt=grpt.cpu().numpy(), nprod=res.nprod)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("name", ["cant", "webbase"])
+def test_two_rank_row_partition(tmp_path, name):
+    import oracle
+    import synth
+    if not torch.cuda.is_available():
+        pytest.fail("needs a GPU")
+    mp.spawn(_worker, args=(2, _port(), name, str(tmp_path)), nprocs=2, join=True)
+    H = synth.config(name, "int").astype(np.float32)
+    r_rpt, r_col, r_val, _ = oracle.spgemm(H, H, np.float32)
+    _, total = oracle.nprod(H, H)
+    sh = [np.load(os.path.join(tmp_path, f"r{p}.npz")) for p in range(2)]
+    assert np.array_equal(sh[0]["splits"], sh[1]["splits"])
+    assert np.array_equal(sh[0]["grpt"], r_rpt)
+    assert np.array_equal(np.concatenate([s["col"] for s in sh]), r_col)
+    assert np.array_equal(np.concatenate([s["val"] for s in sh]), r_val)
+    assert sum(int(s["nprod"]) for s in sh) == total

@@ -225,6 +225,20 @@ def test_duplicates_unsorted(spg):
     check(spg, A, B, np.float64, exact=True, what="dup/unsorted")
 
 
+def test_duplicate_columns_in_b_rows(spg):
+    """Repeated columns inside B rows (legal input) must not race in any accumulation path."""
+    base = synth.banded(3000, 4, 30, 20, seed=8)
+    rng = np.random.default_rng(3)
+    rows = np.repeat(np.arange(base.m), np.diff(base.rpt))
+    extra = rng.integers(0, len(rows), size=len(rows) // 3)
+    B = from_coo(base.m, base.n, np.concatenate([rows, rows[extra]]), np.concatenate([base.col, base.col[extra]]),
+                 dedup=False).with_values("int", 2)
+    A = synth.banded(3000, 4, 30, 20, seed=9).with_values("int", 1)
+    for rh in (0, 1):
+        check(spg, A, B, np.float64, exact=True, opts={"range_hash": rh}, what=f"dup B rows rh={rh}")
+        check(spg, A, B, np.float32, exact=True, opts={"range_hash": rh, "lanes": 4}, what=f"dup B rows vw4 rh={rh}")
+
+
 def test_large_column_indices(spg):
     n = 2**31 - 2
     rng = np.random.default_rng(0)
