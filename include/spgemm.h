@@ -126,9 +126,17 @@ typedef enum {
     SPGEMM_OPT_TIMING = 7,          /* 1 = per-group CUDA-event timing (default 1) */
     SPGEMM_OPT_LONG_ROW = 8,        /* CTA-per-row groups: B rows longer than v are walked by
                                        the whole CTA (0 = auto, -1 = off) */
-    SPGEMM_OPT_RANGE_HASH = 9       /* 1 (default): rows whose column span fits the group's table
+    SPGEMM_OPT_RANGE_HASH = 9,      /* 1 (default): rows whose column span fits the group's table
                                        use the offset hash key - lo_i (collision-free, ordered);
                                        0: the paper's multiplicative hash (Alg. 5) everywhere */
+    SPGEMM_OPT_CLUSTER = 10,        /* 1 (default): rows beyond one SM's shared memory use a
+                                       cluster-per-row table in distributed shared memory before
+                                       the global-memory fallback; 0: straight to global memory */
+    SPGEMM_OPT_CLUSTER_FILL_LIMIT = 11, /* symbolic cluster table: rows with more distinct keys
+                                       than v go to global memory (0 = capacity/2) */
+    SPGEMM_OPT_FLAT = 12            /* product loop: 1 load-balanced flattened (lanes share a batch
+                                       of A non-zeros), 0 VW lanes per A non-zero, -1 auto (1 when
+                                       the mean B row is shorter than 16) */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);
@@ -145,11 +153,12 @@ typedef struct {
     int64_t sym_nprod[SPGEMM_MAX_GROUPS], num_nprod[SPGEMM_MAX_GROUPS];
     int64_t sym_nnza[SPGEMM_MAX_GROUPS], num_nnza[SPGEMM_MAX_GROUPS];
     int64_t num_nnzc[SPGEMM_MAX_GROUPS];
-    int64_t sym_overflow_rows;          /* rows retried in the global-memory table */
+    int64_t sym_overflow_rows;          /* rows that overflowed the one-CTA optimistic table */
     float sym_group_ms[SPGEMM_MAX_GROUPS], num_group_ms[SPGEMM_MAX_GROUPS];
     float setup_ms, symbolic_ms, scan_ms, numeric_ms; /* phases (Figure 5/6 breakdown) */
     int64_t kernel_launches_symbolic, kernel_launches_numeric;
     int64_t workspace_bytes, workspace_peak_bytes;
+    int64_t sym_overflow2_rows;         /* rows that overflowed the cluster table (global memory) */
 } spgemm_stats_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);

@@ -42,12 +42,37 @@ struct Vec16<float> { using T = float4; static __device__ __forceinline__ float4
 template <>
 struct Vec16<double> { using T = double2; static __device__ __forceinline__ double2 zero() { return make_double2(0.0, 0.0); } };
 
+// The product loop of one numeric row: CTA-per-row groups in flat mode use the block-level
+// flattened loop; otherwise the per-sub-group loop plus the CTA pass over deferred long B rows.
+template <int TPR, typename VT, typename F>
+__device__ __forceinline__ void num_products(const NumArgs& a, bool active, int row, int t, int long_len, int* s_list,
+                                             int* s_lcnt, BlockFlat<VT>* bf, long long* ws, F&& f) {
+  const VT* av = static_cast<const VT*>(a.a_val);
+  const VT* bv = static_cast<const VT*>(a.b_val);
+  if constexpr (TPR > 32) {
+    if (a.flat) {
+      for_each_product_block<true, false, VT, TPR>(a.a_rpt, a.a_col, av, a.b_rpt, a.b_col, bv, active, row, t, bf, ws,
+                                                   f, NoStop{});
+      return;
+    }
+  }
+  if (active)
+    products<true, false, VT, TPR>(a.flat, a.a_rpt, a.a_col, av, a.b_rpt, a.b_col, bv, row, t, TPR, a.vw_log2, f,
+                                   NoStop{}, long_len, s_lcnt);
+  if constexpr (TPR > 32) {
+    if (long_len > 0)
+      for_long_products<true, false, VT>(a.a_rpt, a.a_col, av, a.b_rpt, a.b_col, bv, active, row, t, TPR, long_len,
+                                         s_list, s_lcnt, f, NoStop{});
+  }
+}
+
 // One row: (0) init, (a) accumulate, (b) gather into buckets, (c) rank + write.
 // Kp/Vp: the key/value tables (shared or global); Keys/Vals: their probe/add accessors.
 template <typename VT, int TPR, bool GLOBAL, typename Keys, typename Vals, typename SIdx>
 __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, const Keys& K, const Vals& V,
                                         int* Kp, VT* Vp, int* Bc, SIdx* S, unsigned mask, int NB, int* lohi,
-                                        long long* ws, int* s_list, int* s_lcnt, unsigned* wscr) {
+                                        long long* ws, int* s_list, int* s_lcnt, unsigned* wscr,
+                                        BlockFlat<VT>* bf) {
   const int t = Grp<TPR>::lane();
   const unsigned T = mask + 1;
   if (TPR > 32 && t == 0) *s_lcnt = 0;  // pass-1 "deferred a long row" flag (read after a barrier)
@@ -139,15 +164,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
           st_s8(kb + d, 1);
           V.add(d, prod);
         };
-        for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
-                                          static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
-                                          long_len, s_lcnt);
-        if constexpr (TPR > 32) {
-          if (long_len > 0)
-            for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
-                                               a.b_col, static_cast<const VT*>(a.b_val), true, row, t, TPR,
-                                               long_len, s_list, s_lcnt, f, NoStop{});
-        }
+        num_products<TPR>(a, true, row, t, long_len, s_list, s_lcnt, bf, ws, f);
         Grp<TPR>::sync();
         // in-order compaction: thread owns a contiguous run of flag words
         const int pw = (words + TPR - 1) / TPR;
@@ -189,16 +206,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
       V.add(s, prod);
     };
     const int long_len = TPR > 32 ? a.long_len : 0;
-    if (active)
-      for_each_product<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
-                                        static_cast<const VT*>(a.b_val), row, t, TPR, a.vw_log2, f, NoStop{},
-                                        long_len, s_lcnt);
-    if constexpr (TPR > 32) {
-      if (long_len > 0)
-        for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
-                                           static_cast<const VT*>(a.b_val), active, row, t, TPR, long_len, s_list,
-                                           s_lcnt, f, NoStop{});
-    }
+    num_products<TPR>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f);
   }
   Grp<TPR>::sync();
 
@@ -432,7 +440,13 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   constexpr int RPB = BS / TPR;
   __shared__ int s_lohi[2 * RPB];
   __shared__ int s_list[TPR > 32 ? kLongChunk : 1], s_lcnt;
-  __shared__ unsigned s_wscr[TPR > 32 ? (TPR / 32) * 2 * kWarpBitmapWords<TPR> : 1];  // bucket bitmap+prefix
+  // per-warp bucket bitmap+prefix of the (c4) sort, aliased with the block-flat product scratch
+  // (used in different phases of a row; separated by barriers)
+  constexpr int kWscrBytes = TPR > 32 ? (TPR / 32) * 8 * kWarpBitmapWords<TPR> : 4;
+  constexpr int kAuxBytes = TPR > 32 ? (kWscrBytes > (int)sizeof(BlockFlat<VT>) ? kWscrBytes : (int)sizeof(BlockFlat<VT>))
+                                     : 4;
+  __shared__ __align__(16) unsigned char s_aux[kAuxBytes];
+  unsigned* s_wscr = reinterpret_cast<unsigned*>(s_aux);
   constexpr int NB = num_nbuckets(T);
   constexpr int RB = num_row_bytes<VT>(T, UPPER);
   const int g = threadIdx.x / TPR;
@@ -445,13 +459,14 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : 0;
   num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
-                          s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr);
+                          s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr, reinterpret_cast<BlockFlat<VT>*>(s_aux));
 }
 
 template <typename VT>
 __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_lohi[2];
+  __shared__ BlockFlat<VT> s_bf;
   __shared__ int s_list[kLongChunk], s_lcnt;
   unsigned char* slab = static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride;
   VT* Vp = reinterpret_cast<VT*>(slab);
@@ -465,7 +480,7 @@ __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
     while (T < 2 * n) T <<= 1;
     if (T > a.slab_T) T = a.slab_T;
     num_row<VT, 1024, true>(a, true, row, GKeys{Kp}, GVals<VT>{Vp}, Kp, Vp, Bc, S, (unsigned)(T - 1), 0,
-                      s_lohi, ws, s_list, &s_lcnt, nullptr);
+                            s_lohi, ws, s_list, &s_lcnt, nullptr, &s_bf);
   }
 }
 
@@ -473,7 +488,9 @@ template <typename VT, int T, int TPR, int BS, long long UPPER>
 cudaError_t launch_num(cudaStream_t s, const NumArgs& a) {
   constexpr int RPB = BS / TPR;
   constexpr int smem = RPB * num_row_bytes<VT>(T, UPPER);
-  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 + (TPR > 32 ? TPR / 32 * 8 * kWarpBitmapWords<TPR> : 4) <= kSmemLimit,
+  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 +
+                    (TPR > 32 ? (TPR / 32 * 8 * kWarpBitmapWords<TPR> > (int)sizeof(BlockFlat<VT>)
+                                     ? TPR / 32 * 8 * kWarpBitmapWords<TPR> : (int)sizeof(BlockFlat<VT>)) : 4) <= kSmemLimit,
                 "numeric table too large");
   static bool configured = false;
   if (!configured) {

@@ -13,6 +13,8 @@
 // table and aborts a row once it has found `fill_limit` distinct keys; the row index is
 // recorded and the row is recounted in a global-memory table sized from its n_prod
 // by k_sym_global.
+#include <type_traits>
+
 #include "spgemm_internal.cuh"
 
 namespace spg {
@@ -23,10 +25,33 @@ struct NoStop {
   __device__ __forceinline__ bool operator()() const { return false; }
 };
 
+// The product loop of one symbolic row: CTA-per-row groups in flat mode use the block-level
+// flattened loop; otherwise the per-sub-group loop plus the CTA pass over deferred long B rows.
+template <bool STOP, int TPR, typename F, typename S>
+__device__ __forceinline__ void sym_products(const SymArgs& a, bool active, int row, int t, int long_len,
+                                             int* s_list, int& s_lcnt, BlockFlat<int>* bf, long long* ws, F&& f,
+                                             S&& stop) {
+  if constexpr (TPR > 32) {
+    if (a.flat) {
+      for_each_product_block<false, STOP, int, TPR>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row,
+                                                    t, bf, ws, f, stop);
+      return;
+    }
+  }
+  if (active)
+    products<false, STOP, int, TPR>(a.flat, a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
+                                    a.vw_log2, f, stop, long_len, &s_lcnt);
+  if constexpr (TPR > 32) {
+    if (long_len > 0)
+      for_long_products<false, STOP, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t, TPR,
+                                          long_len, s_list, &s_lcnt, f, stop);
+  }
+}
+
 // One row (all TPR threads of its row group call it; the table is the group's slice).
 template <int T, int TPR, bool OPT>
 __device__ __forceinline__ void sym_row(const SymArgs& a, bool active, int row, int t, int* table, long long* ws,
-                                        int& s_cnt, int& s_abort, int& s_lcnt, int* s_list) {
+                                        int& s_cnt, int& s_abort, int& s_lcnt, int* s_list, BlockFlat<int>* bf) {
   // Range-offset hash: when the row's column span R fits 4*T bytes the table
   // is a byte-flag array indexed by key - lo_i (collision-free; idempotent plain stores, no
   // atomics, conflict-free for consecutive keys); the count is the number of set flags.
@@ -61,14 +86,7 @@ __device__ __forceinline__ void sym_row(const SymArgs& a, bool active, int row, 
       if (bitmap) red_or_s(tb + 4u * (d >> 5), 1u << (d & 31));
       else st_s8(tb + d, 1);
     };
-    if (active)
-      for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
-                                          a.vw_log2, f, NoStop{}, long_len, &s_lcnt);
-    if constexpr (TPR > 32) {
-      if (long_len > 0)
-        for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
-                                             TPR, long_len, s_list, &s_lcnt, f, NoStop{});
-    }
+    sym_products<false, TPR>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f, NoStop{});
     Grp<TPR>::sync();
     for (int w = t; w < words; w += TPR) cnt += __popc((unsigned)table[w]);  // 0/1 bytes or bits
     const int tot = Grp<TPR>::sum32(cnt, reinterpret_cast<int*>(ws));
@@ -83,26 +101,14 @@ __device__ __forceinline__ void sym_row(const SymArgs& a, bool active, int row, 
       probe(K, T - 1, key, ins);
       if (ins && atomicAdd(&s_cnt, 1) + 1 >= a.fill_limit) s_abort = 1;
     };
-    if (active)
-      for_each_product<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
-                                         a.vw_log2, f, stop, long_len, &s_lcnt);
-    if (long_len > 0)
-      for_long_products<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
-                                          TPR, long_len, s_list, &s_lcnt, f, stop);
+    sym_products<true, TPR>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f, stop);
   } else {
     auto f = [&](int key, int) {
       bool ins;
       probe(K, T - 1, key, ins);
       cnt += ins;
     };
-    if (active)
-      for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, TPR,
-                                          a.vw_log2, f, NoStop{}, long_len, &s_lcnt);
-    if constexpr (TPR > 32) {
-      if (long_len > 0)
-        for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t,
-                                             TPR, long_len, s_list, &s_lcnt, f, NoStop{});
-    }
+    sym_products<false, TPR>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f, NoStop{});
   }
   if constexpr (OPT) {
     __syncthreads();
@@ -126,6 +132,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_cnt, s_abort, s_lcnt;
   __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
+  __shared__ std::conditional_t<(TPR > 32), BlockFlat<int>, int> s_bf_store;  // only CTA groups need it
   constexpr int RPB = BS / TPR;
   static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
   const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
@@ -133,7 +140,8 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   const long long ridx = (long long)blockIdx.x * RPB + g;
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : -1;
-  sym_row<T, TPR, OPT>(a, active, row, t, table, ws, s_cnt, s_abort, s_lcnt, s_list);
+  sym_row<T, TPR, OPT>(a, active, row, t, table, ws, s_cnt, s_abort, s_lcnt, s_list,
+                       reinterpret_cast<BlockFlat<int>*>(&s_bf_store));
 }
 
 // Global-memory table per CTA (slab of slab_T ints), one row at a time; table size
@@ -142,12 +150,13 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
 __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_list[kLongChunk], s_lcnt;
+  __shared__ BlockFlat<int> s_bf;
   int* table = a.slab + (long long)blockIdx.x * a.slab_T;
   const long long nA = a.nrows;
-  const long long nB = a.dev_count ? (long long)*a.dev_count : 0;
+  const long long nB = a.dev_count2 ? (long long)*a.dev_count2 : 0;
   const int t = threadIdx.x;
   for (long long i = blockIdx.x; i < nA + nB; i += gridDim.x) {
-    const int row = i < nA ? a.rows[i] : a.overflow_rows[i - nA];
+    const int row = i < nA ? a.rows[i] : a.overflow2_rows[i - nA];
     const long long cap = a.nprod[row] < a.n ? a.nprod[row] : a.n;
     long long T = 64;
     while (T < 2 * cap) T <<= 1;
@@ -163,11 +172,16 @@ __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
       probe(K, (unsigned)(T - 1), key, ins);
       cnt += ins;
     };
-    for_each_product<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, 1024,
+    if (a.flat) {
+      for_each_product_block<false, false, int, 1024>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row,
+                                                      t, &s_bf, ws, f, NoStop{});
+    } else {
+      products<false, false, int, 1024>(false, a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, row, t, 1024,
                                         a.vw_log2, f, NoStop{}, a.long_len, &s_lcnt);
-    if (a.long_len > 0)
-      for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
-                                           a.long_len, s_list, &s_lcnt, f, NoStop{});
+      if (a.long_len > 0)
+        for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
+                                             a.long_len, s_list, &s_lcnt, f, NoStop{});
+    }
     const long long tot = Grp<1024>::sum(cnt, ws);
     if (t == 0) a.c_cnt[row] = tot;
     __syncthreads();

@@ -66,6 +66,9 @@ struct spgemm_ctx {
   int sym_min_group = -1, num_min_group = -1, fill_limit = 0, use_streams = 1, validate = 0, lanes = 0;
   int long_len = 0;  // 0 auto, -1 off
   int range_hash = 1;  // 1: range-offset hash where a row's column span fits
+  int cluster_fill = 0;  // symbolic cluster table fill limit (0 = capacity / 2)
+  int use_cluster = 1;   // 0: rows beyond one CTA go straight to global memory (ablation)
+  int flat = -1;         // load-balanced flattened product loop: -1 auto (mean B row < 16), 0, 1
   int timing = 1;
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -76,7 +79,7 @@ struct spgemm_ctx {
   const int32_t *a_col = nullptr, *b_col = nullptr;
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
-  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, slab_sym, bmm, rlohi;
+  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi;
   bool perm2_ready = false;
   bool group_sums_done = false;  // per-group n_prod/nnz sums (computed on demand by get_stats)
   DevAcc* hacc = nullptr;      // pinned
@@ -138,8 +141,8 @@ void buf_free(spgemm_handle_t h, Buf& b) {
 }
 
 void release_state(spgemm_handle_t h) {
-  Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow, &h->slab_sym,
-                &h->bmm, &h->rlohi};
+  Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow,
+                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi};
   for (Buf* b : all) buf_free(h, *b);
   h->state = 0;
   h->perm2_ready = false;
@@ -211,6 +214,11 @@ int auto_vw_log2(spgemm_handle_t h) {
 }
 
 // CTA-per-row kernels hand B rows longer than this to the whole CTA (load balance).
+bool flat_of(spgemm_handle_t h) {
+  if (h->flat >= 0) return h->flat != 0;
+  return h->k > 0 && (double)h->nnzb / (double)h->k < 16.0;
+}
+
 int long_len_of(spgemm_handle_t h) {
   if (h->long_len < 0) return 0;
   if (h->long_len > 0) return h->long_len;
@@ -360,6 +368,13 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->ws_budget = v; break;
     case SPGEMM_OPT_TIMING: h->timing = v ? 1 : 0; break;
     case SPGEMM_OPT_RANGE_HASH: h->range_hash = v ? 1 : 0; break;
+    case SPGEMM_OPT_CLUSTER: h->use_cluster = v ? 1 : 0; break;
+    case SPGEMM_OPT_FLAT:
+      if (v < -1 || v > 1) return fail(h, SPGEMM_ERR_INVALID_ARG, "FLAT must be -1, 0 or 1");
+      h->flat = (int)v; break;
+    case SPGEMM_OPT_CLUSTER_FILL_LIMIT:
+      if (v < 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "CLUSTER_FILL_LIMIT < 0");
+      h->cluster_fill = (int)std::min<int64_t>(v, 1 << 30); break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -446,15 +461,19 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   // (3) symbolic hash counting per group
   const long long n_opt = (long long)h->snap1.sym_rows[kSymOptimistic];
   const long long n_glob = (long long)h->snap1.sym_rows[kSymGlobal];
-  if (n_opt > 0) ALLOC(h->overflow, sizeof(int32_t) * n_opt);
+  if (n_opt > 0) {
+    ALLOC(h->overflow, sizeof(int32_t) * n_opt);
+    ALLOC(h->overflow2, sizeof(int32_t) * n_opt);
+  }
   int glob_grid = 0;
   long long slab_T = 0;
-  if (n_opt + n_glob > 0) {
+  if (n_opt + n_glob > 0) {  // global tables: forced-global rows and rows beyond the cluster table
     const long long cap = std::min<long long>((long long)h->snap1.max_nprod, n);
     slab_T = std::max<long long>(64, next_pow2(2 * std::max<long long>(cap, 1)));
     const long long per = slab_T * 4;
     const long long by_budget = std::max<long long>(1, h->ws_budget / per);
-    glob_grid = (int)std::min<long long>({n_opt + n_glob, 2LL * h->num_sms, by_budget});
+    const long long want = n_glob + (h->use_cluster ? std::min<long long>(n_opt, 32) : n_opt);
+    glob_grid = (int)std::min<long long>({want, 2LL * h->num_sms, by_budget});
     ALLOC(h->slab_sym, (size_t)(glob_grid * per));
   }
   SymArgs sa{};
@@ -462,6 +481,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.c_cnt = c_rpt + 1;
   sa.vw_log2 = h->vw_log2;
   sa.long_len = long_len_of(h);
+  sa.flat = flat_of(h) ? 1 : 0;
   sa.rlohi = static_cast<const int2*>(h->rlohi.p);
   sa.overflow_rows = static_cast<int32_t*>(h->overflow.p);
   sa.overflow_count = &dacc->overflow_count;
@@ -488,7 +508,20 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       SymArgs gb = sa;
       gb.rows = perm1 + off1.off[kSymGlobal];
       gb.nrows = n_glob;
-      gb.dev_count = &dacc->overflow_count;
+      if (h->use_cluster) {  // overflow rows -> cluster DSMEM table -> (overflow2) global table
+        SymArgs cb = sa;
+        cb.nrows = 0;
+        const int climit = h->cluster_fill > 0 ? std::min(h->cluster_fill, cluster_capacity_sym() / 2)
+                                               : cluster_capacity_sym() / 2;
+        CK(launch_symbolic_cluster(s, cb, nullptr, &dacc->overflow_count, static_cast<int32_t*>(h->overflow2.p),
+                                   &dacc->overflow2_count, climit, (int)n_opt));
+        ++launches;
+        gb.overflow2_rows = static_cast<const int32_t*>(h->overflow2.p);
+        gb.dev_count2 = &dacc->overflow2_count;
+      } else {
+        gb.overflow2_rows = static_cast<const int32_t*>(h->overflow.p);
+        gb.dev_count2 = &dacc->overflow_count;
+      }
       CK(launch_symbolic_global(s, gb, glob_grid));
       ++launches;
     }
@@ -501,7 +534,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
     SymArgs gb = sa;
     gb.rows = perm1 + off1.off[kSymGlobal];
     gb.nrows = n_glob;
-    gb.dev_count = nullptr;
+    gb.dev_count2 = nullptr;
     CK(launch_symbolic_global(s, gb, glob_grid));
     ++launches;
     if (h->timing) CK(cudaEventRecord(h->gstop[0][kSymGlobal], s));
@@ -537,6 +570,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   }
   h->group_sums_done = false;
   st.sym_overflow_rows = h->snap2.overflow_count;
+  st.sym_overflow2_rows = h->snap2.overflow2_count;
   st.kernel_launches_symbolic = launches;
   h->state = 1;
   return SPGEMM_OK;
@@ -579,10 +613,27 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.c_rpt = h->c_rpt; na.c_col = c_col; na.c_val = c_val;
     na.vw_log2 = h->vw_log2;
     na.long_len = long_len_of(h);
+    na.flat = flat_of(h) ? 1 : 0;
     na.rlohi = static_cast<const int2*>(h->rlohi.p);
     na.priv_ok = h->snap1.b_unsorted ? 0 : 1;
     na.err_flags = &dacc->err_flags;
-    Buf slab;
+    Buf slab, slab_c;
+    // cluster groups (clusters of 2/4/8 CTAs): bitmap + prefix scratch per resident cluster
+    const long long cwords = h->n / 32 + 2;
+    const long long cstride = (2 * cwords * 4 + 255) & ~255LL;
+    long long ccount[3] = {0, 0, 0}, ctotal = 0;
+    for (int c = 0; c < 3; ++c) {
+      const long long rows_c = (long long)h->snap2.num_rows[kNumCluster + c];
+      if (rows_c == 0) continue;
+      int nc = 0;
+      CK(launch_numeric_cluster(h->stream, fp64, 2 << c, na, &nc));
+      ccount[c] = std::min<long long>(nc, rows_c);
+      ctotal += ccount[c];
+    }
+    if (ctotal > 0) {
+      s = buf_alloc(h, slab_c, (size_t)(ctotal * cstride));
+      if (s != SPGEMM_OK) return s;
+    }
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
     int glob_grid = 0;
     if (n_glob > 0) {
@@ -607,14 +658,27 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
       NumArgs ga = na;
       ga.rows = perm2 + off2.off[g];
       ga.nrows = rows;
-      if (g == kNumGlobal) CK(launch_numeric_global(st, fp64, ga, glob_grid));
-      else CK(launch_numeric_group(st, g, fp64, ga));
+      if (g == kNumGlobal) {
+        CK(launch_numeric_global(st, fp64, ga, glob_grid));
+      } else if (g >= kNumCluster && g < kNumCluster + 3) {
+        const int c = g - kNumCluster;
+        long long before = 0;
+        for (int q = 0; q < c; ++q) before += ccount[q];
+        NumArgs gc = ga;
+        gc.slab = static_cast<unsigned char*>(slab_c.p) + before * cstride;
+        gc.bitmap_words = cwords;
+        gc.slab_stride = cstride;
+        CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
+      } else {
+        CK(launch_numeric_group(st, g, fp64, ga));
+      }
       h->stats.kernel_launches_numeric += 1;
       if (h->timing) CK(cudaEventRecord(h->gstop[1][g], st));
       h->gtimed[1][g] = true;
     }
     CK(join(h));
     buf_free(h, slab);
+    buf_free(h, slab_c);
   }
   if (h->timing) CK(cudaEventRecord(h->ev[5], h->stream));
   return SPGEMM_OK;

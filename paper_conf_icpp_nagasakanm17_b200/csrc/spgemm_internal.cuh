@@ -53,15 +53,24 @@ constexpr int kSymGlobal = 11;
 constexpr int kNumSymGroups = 12;   // including global
 
 // Phase 2 (numeric), key = nnz_i.  Same bounds for fp32 and fp64 (fp64 sizes the smem).
+// Groups 10-12 = cluster-per-row (DSMEM of 2/4/8 CTAs, kernels_cluster.cu; load factor up to 3/4
+// so an 8-CTA cluster covers the heaviest rows of the graph configs), 13 = global.
+constexpr int kClusterSize = 8;
+constexpr int kClusterSymSlots = 32768;  // int keys per CTA (128 KB)
+constexpr int kClusterNumSlots = 16384;  // key+value slots per CTA (128 KB fp32, 192 KB fp64)
 constexpr GroupSpec kNumGroups[] = {
     {8, 16, 4, 256},         {16, 32, 8, 256},         {64, 128, 16, 256},
     {128, 256, 32, 256},     {256, 512, 64, 64},       {512, 1024, 128, 128},
     {1024, 2048, 256, 256},  {2048, 4096, 512, 512},   {4096, 8192, 1024, 1024},
     {8192, 16384, 1024, 1024},
+    {2 * kClusterNumSlots * 3 / 4, 2 * kClusterNumSlots, 2 * 1024, 1024},   // cluster of 2 CTAs
+    {4 * kClusterNumSlots * 3 / 4, 4 * kClusterNumSlots, 4 * 1024, 1024},   // cluster of 4 CTAs
+    {8 * kClusterNumSlots * 3 / 4, 8 * kClusterNumSlots, 8 * 1024, 1024},   // cluster of 8 CTAs
 };
-constexpr int kNumNumBounds = 10;
-constexpr int kNumGlobal = 10;
-constexpr int kNumNumGroups = 11;
+constexpr int kNumNumBounds = 13;
+constexpr int kNumCluster = 10;  // groups 10, 11, 12: clusters of 2, 4, 8 CTAs
+constexpr int kNumGlobal = 13;
+constexpr int kNumNumGroups = 14;
 
 // Numeric per-row shared-memory layout: vals[T] | keys[T] | bucket[NB+1] | sidx[upper] ,
 // NB = T/2 (T/8 for the largest table) buckets for the bucket-rank sort.
@@ -82,6 +91,7 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   unsigned long long num_nnzc[kMaxGroups];
   long long nnzc;
   int overflow_count;
+  int overflow2_count;  // rows that overflowed the cluster table too (-> global memory)
   int err_flags;  // bit0 invalid input, bit1 numeric row count mismatch
   int b_unsorted;  // some B row is not strictly increasing (disables private accumulators)
   int cursor[2][kMaxGroups];
@@ -252,6 +262,152 @@ __device__ __forceinline__ void for_each_product(const int64_t* __restrict__ a_r
   }
 }
 
+// Load-balanced variant for short B rows (graphs): groups of G lanes (G = min(TPR, 32)) take
+// batches of G consecutive A non-zeros, scan their B-row lengths, and lane l handles products
+// l, l+G, l+2G, ... of the concatenated batch, finding its A non-zero by a log2(G)-step shuffle
+// binary search — every lane does the same work whatever the B-row lengths (the VW-per-entry
+// loop leaves most lanes idle on 2-4-entry rows and serialises on 30-60-entry rows).
+template <bool NUM, bool CHECK_STOP, typename VT, int G, typename F, typename S>
+__device__ __forceinline__ void for_each_product_flat(const int64_t* __restrict__ a_rpt,
+                                                      const int32_t* __restrict__ a_col,
+                                                      const VT* __restrict__ a_val,
+                                                      const int64_t* __restrict__ b_rpt,
+                                                      const int32_t* __restrict__ b_col,
+                                                      const VT* __restrict__ b_val, int row, int t, int tpr,
+                                                      F&& f, S&& stop, int long_len, int* deferred) {
+  const long long a0 = __ldg(a_rpt + row);
+  const int na = (int)(__ldg(a_rpt + row + 1) - a0);
+  const int32_t* __restrict__ ac = opaque(a_col + a0);
+  const VT* __restrict__ avp = NUM ? opaque(a_val + a0) : nullptr;
+  const int gl = t % G, gi = t / G, ng = tpr / G;
+  const unsigned gm = G >= 32 ? 0xffffffffu : (((1u << G) - 1u) << ((threadIdx.x & 31) & ~(G - 1)));
+  for (int base = gi * G; base < na; base += ng * G) {  // uniform within the group
+    const int j = base + gl;
+    int len = 0;
+    long long b0 = 0;
+    VT av = VT(0);
+    if (j < na) {
+      const int kk = __ldg(ac + j);
+      if (NUM) av = __ldg(avp + j);
+      b0 = __ldg(b_rpt + kk);
+      len = (int)(__ldg(b_rpt + kk + 1) - b0);
+      if (long_len > 0 && len > long_len) {  // deferred to for_long_products
+        len = 0;
+        if (deferred) *deferred = 1;
+      }
+    }
+    int incl = len;
+#pragma unroll
+    for (int d = 1; d < G; d <<= 1) {
+      const int y = __shfl_up_sync(gm, incl, d, G);
+      if (gl >= d) incl += y;
+    }
+    const int total = __shfl_sync(gm, incl, G - 1, G);
+    for (int p0 = 0; p0 < total; p0 += G) {
+      const int p = p0 + gl;
+      int e = 0;
+#pragma unroll
+      for (int st = G / 2; st > 0; st >>= 1)
+        if (__shfl_sync(gm, incl, e + st - 1, G) <= p) e += st;
+      const int ie = __shfl_sync(gm, incl, e, G);
+      const int le = __shfl_sync(gm, len, e, G);
+      const long long be = __shfl_sync(gm, b0, e, G);
+      const VT ae = NUM ? __shfl_sync(gm, av, e, G) : VT(0);
+      if (p < total) {
+        const long long q = be + (p - (ie - le));
+        const int key = __ldg(b_col + q);
+        const VT v = NUM ? __ldg(b_val + q) : VT(0);
+        if (!(CHECK_STOP && stop())) f(key, ae * v);
+      }
+    }
+    if constexpr (CHECK_STOP) {
+      if (__any_sync(gm, stop())) return;
+    }
+  }
+}
+
+// CTA-level flattened loop for CTA-per-row groups (every thread of the CTA must call it): the
+// row's A non-zeros are taken in chunks of kFlatChunk; their metadata and the inclusive scan of
+// their B-row lengths go to shared memory (BlockFlat), and all tpr threads stride the chunk's
+// concatenated products, each locating its A non-zero by binary search over the scan.  Equal
+// work per thread whatever the B-row lengths — no long-row deferral needed.
+constexpr int kFlatChunk = 256;
+template <int TPR>
+struct Grp;  // row-group collectives (defined below)
+template <typename VT>
+struct BlockFlat {
+  long long b0[kFlatChunk];
+  int incl[kFlatChunk];
+  VT av[kFlatChunk];
+};
+template <bool NUM, bool CHECK_STOP, typename VT, int TPR, typename F, typename S>
+__device__ __forceinline__ void for_each_product_block(const int64_t* __restrict__ a_rpt,
+                                                       const int32_t* __restrict__ a_col,
+                                                       const VT* __restrict__ a_val,
+                                                       const int64_t* __restrict__ b_rpt,
+                                                       const int32_t* __restrict__ b_col,
+                                                       const VT* __restrict__ b_val, bool active, int row, int t,
+                                                       BlockFlat<VT>* sh, long long* ws, F&& f, S&& stop,
+                                                       int part = 0, int nparts = 1) {
+  static_assert(TPR > 32, "CTA-level loop");
+  constexpr int CH = TPR < kFlatChunk ? TPR : kFlatChunk;
+  constexpr int tpr = TPR;
+  const long long a0 = active ? __ldg(a_rpt + row) : 0;
+  const int na = active ? (int)(__ldg(a_rpt + row + 1) - a0) : 0;  // CTA-uniform
+  const int32_t* __restrict__ ac = a_col + a0;
+  for (int c = part * CH; c < na; c += nparts * CH) {
+    const int cn = min(CH, na - c);
+    int len = 0;
+    if (t < cn) {
+      const int kk = __ldg(ac + c + t);
+      const long long b0 = __ldg(b_rpt + kk);
+      len = (int)(__ldg(b_rpt + kk + 1) - b0);
+      sh->b0[t] = b0;
+      if (NUM) sh->av[t] = __ldg(a_val + a0 + c + t);
+    }
+    long long tot;
+    const long long ex = Grp<TPR>::excl_scan(t < cn ? len : 0, &tot, ws);  // block scan
+    if (t < cn) sh->incl[t] = (int)(ex + len);
+    __syncthreads();
+    const int P = (int)tot;
+#pragma unroll 1
+    for (int p = t; p < P; p += tpr) {
+      int lo = 0, hi = cn - 1;  // first e with incl[e] > p
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (sh->incl[mid] <= p) lo = mid + 1; else hi = mid;
+      }
+      const int e = lo;
+      const int start = e ? sh->incl[e - 1] : 0;
+      const long long q = sh->b0[e] + (p - start);
+      const int key = __ldg(b_col + q);
+      const VT v = NUM ? __ldg(b_val + q) : VT(0);
+      if (CHECK_STOP && stop()) break;
+      f(key, NUM ? sh->av[e] * v : VT(0));
+    }
+    __syncthreads();
+  }
+}
+
+// Dispatch: flattened load-balanced loop (flat, short B rows) or the VW-lanes-per-A-entry loop.
+// GMAX: the row group's lane count (TPR).  CTA-per-row groups in flat mode use
+// for_each_product_block instead (see the callers).
+template <bool NUM, bool CHECK_STOP, typename VT, int GMAX, typename F, typename S>
+__device__ __forceinline__ void products(bool flat, const int64_t* __restrict__ a_rpt,
+                                         const int32_t* __restrict__ a_col, const VT* __restrict__ a_val,
+                                         const int64_t* __restrict__ b_rpt, const int32_t* __restrict__ b_col,
+                                         const VT* __restrict__ b_val, int row, int t, int tpr, int vwl, F&& f,
+                                         S&& stop, int long_len, int* deferred) {
+  // flat only for row groups of <= 32 lanes: in CTA-per-row groups, batches of 32 consecutive A
+  // non-zeros per warp leave most warps idle on rows with a few hundred non-zeros (measured)
+  if (flat && GMAX <= 32)
+    for_each_product_flat<NUM, CHECK_STOP, VT, (GMAX < 32 ? GMAX : 32)>(a_rpt, a_col, a_val, b_rpt, b_col, b_val, row,
+                                                                       t, tpr, f, stop, long_len, deferred);
+  else
+    for_each_product<NUM, CHECK_STOP, VT>(a_rpt, a_col, a_val, b_rpt, b_col, b_val, row, t, tpr, vwl, f, stop,
+                                          long_len, deferred);
+}
+
 // Second pass (CTA-wide, every thread of the CTA must call it): the A row is rescanned in
 // chunks of kLongChunk entries; entries whose B row is longer than long_len go to a shared
 // list, and all tpr threads stride each listed B row (unrolled by 2).  s_list: kLongChunk
@@ -264,7 +420,7 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
                                                   const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                   const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
                                                   bool active, int row, int t, int tpr, int long_len, int* s_list,
-                                                  int* s_cnt, F&& f, S&& stop) {
+                                                  int* s_cnt, F&& f, S&& stop, int part = 0, int nparts = 1) {
   const long long a0 = active ? __ldg(a_rpt + row) : 0;
   const int32_t* __restrict__ ac = a_col + a0;
   __syncthreads();  // s_cnt doubles as the "some sub-group deferred a row" flag of pass 1
@@ -274,11 +430,16 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
   if (t == 0) *s_cnt = 0;
   __syncthreads();
   for (int c = 0; c < na; c += kLongChunk) {  // na is CTA-uniform
+    bool added = false;
     for (int e = t; e < kLongChunk && c + e < na; e += tpr) {
+      if (nparts > 1 && (c + e) % nparts != part) continue;  // cluster: CTA `part` takes its share
       const int kk = __ldg(ac + c + e);
-      if (__ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk) > long_len) s_list[atomicAdd(s_cnt, 1)] = c + e;
+      if (__ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk) > long_len) {
+        s_list[atomicAdd(s_cnt, 1)] = c + e;
+        added = true;
+      }
     }
-    __syncthreads();
+    if (__syncthreads_count(added) == 0) continue;  // no long row in this chunk: one barrier
     const int n = *s_cnt;
     for (int i = 0; i < n; ++i) {
       const int j = s_list[i];
@@ -456,12 +617,15 @@ struct SymArgs {
   int64_t* c_cnt;          // c_rpt + 1: per-row nnz written here (scanned later)
   int vw_log2;             // lanes per B row = 1 << vw_log2 (Alg. 3/4 generalised)
   int long_len;            // CTA-per-row groups: B rows longer than this are walked by the CTA
+  int flat;                // 1: load-balanced flattened product loop (short B rows)
   const int2* rlohi;       // column span [lo_i, hi_i] of each row of C, or null (paper hash only)
   // optimistic group
   int32_t* overflow_rows; int* overflow_count; int fill_limit;
   // global fallback
   int* slab; long long slab_T; const int64_t* nprod; long long n;
   const int* dev_count;    // extra rows from overflow list (device count), may be null
+  const int32_t* overflow2_rows;  // global kernel: rows that overflowed the cluster table
+  const int* dev_count2;
 };
 
 struct NumArgs {
@@ -471,6 +635,7 @@ struct NumArgs {
   const int64_t* c_rpt; int32_t* c_col; void* c_val;
   int vw_log2;
   int long_len;
+  int flat;                // 1: load-balanced flattened product loop (short B rows)
   const int2* rlohi;       // column span of each row of C, or null (paper hash only)
   int priv_ok;             // B rows strictly increasing: private per-sub-group accumulators allowed
   int* err_flags;
@@ -500,5 +665,10 @@ cudaError_t launch_symbolic_group(cudaStream_t s, int group, const SymArgs& a, i
 cudaError_t launch_symbolic_global(cudaStream_t s, const SymArgs& a, int grid);
 cudaError_t launch_numeric_group(cudaStream_t s, int group, bool fp64, const NumArgs& a);
 cudaError_t launch_numeric_global(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
+cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
+                                    int32_t* overflow2, int* count2, int fill_limit, int max_rows);
+cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);
+int cluster_capacity_sym();
+int cluster_capacity_num();
 
 }  // namespace spg

@@ -134,7 +134,7 @@ def test_forced_symbolic_group(spg, group, range_hash):
 
 
 @pytest.mark.parametrize("range_hash", [0, 1])
-@pytest.mark.parametrize("group", list(range(0, 11)))
+@pytest.mark.parametrize("group", list(range(0, 14)))
 def test_forced_numeric_group(spg, group, range_hash):
     for A in (_mixed_small(), _banded_small()):
         ref = oracle.spgemm(A, A, np.float32)
@@ -150,11 +150,41 @@ def test_paper_hash_only(spg, config):
 
 
 def test_overflow_retry_in_global_memory(spg):
+    """Optimistic one-CTA table -> cluster DSMEM table -> global table (PAPER.md:155 chain)."""
     A = _mixed_small()
     ref = oracle.spgemm(A, A, np.float64)
     got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16, "range_hash": 0})
-    assert got[3]["sym_overflow_rows"] > 0
-    assert_parity(got, ref, np.float64, what="overflow")
+    assert got[3]["sym_overflow_rows"] > 0 and got[3]["sym_overflow2_rows"] == 0
+    assert_parity(got, ref, np.float64, what="overflow -> cluster")
+    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16, "range_hash": 0,
+                                          "cluster_fill_limit": 40})
+    assert got[3]["sym_overflow2_rows"] > 0
+    assert_parity(got, ref, np.float64, what="overflow -> cluster -> global")
+    got = run_gpu(spg, A, A, np.float64, {"sym_min_group": 10, "sym_fill_limit": 16, "range_hash": 0, "cluster": 0})
+    assert_parity(got, ref, np.float64, what="overflow -> global (cluster off)")
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("group", [10, 11, 12])
+def test_cluster_numeric_rows(spg, dtype, group):
+    """Every row through a cluster-per-row numeric kernel (DSMEM table over 2/4/8 CTAs)."""
+    for A in (_mixed_small(), _banded_small(), synth.config("poisson64")):
+        ref = oracle.spgemm(A.astype(dtype), A.astype(dtype), dtype)
+        got = run_gpu(spg, A, A, dtype, {"num_min_group": group})
+        assert got[3]["num_rows"][group] == (np.diff(ref[0]) > 0).sum()
+        assert_parity(got, ref, dtype, what=f"{A.name} cluster-{2 << (group - 10)} numeric")
+
+
+@pytest.mark.parametrize("flat", [0, 1])
+@pytest.mark.parametrize("group", [0, 3, 5, 8, 10, 13])
+def test_flat_and_vw_loops(spg, flat, group):
+    """Both product loops (load-balanced flattened / VW lanes per A entry) in every kernel family."""
+    for A in (_mixed_small(), _banded_small()):
+        ref = oracle.spgemm(A, A, np.float32)
+        for opts in ({"num_min_group": group}, {"sym_min_group": min(group, 11), "range_hash": 0},
+                     {"sym_min_group": 10, "sym_fill_limit": 16, "range_hash": 0}):
+            got = run_gpu(spg, A, A, np.float32, dict(opts, flat=flat))
+            assert_parity(got, ref, np.float32, what=f"{A.name} {opts} flat={flat}")
 
 
 @pytest.mark.parametrize("lanes", [1, 2, 4, 8, 16, 32])
