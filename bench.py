@@ -202,7 +202,9 @@ def run_ours(args):
     tdt = torch.float32 if dt == np.float32 else torch.float64
     vbytes = 4 if dt == np.float32 else 8
     h = P.Handle(dev)
-    h.set_option("lanes", args.lanes).set_option("streams", args.streams)
+    # per-group kernel events over the timed region (timing=2 runs the group kernels eagerly; the
+    # CUDA-graph replay mode is timed separately below and reported as `graph_replay`)
+    h.set_option("lanes", args.lanes).set_option("streams", args.streams).set_option("timing", 2)
     dA = P.CsrMatrix.from_host(A, dev, tdt)
     stream = h.stream
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
@@ -269,6 +271,29 @@ def run_ours(args):
                 "launch_ms": k_ms, "share_of_step": k_ms / (tot_ms / args.steps),
                 "algorithmic_bytes_per_launch": bytes_alg, "peak_source": peak_src}
 
+    # the same step with the captured phase segments replayed as CUDA graphs (timing=1)
+    h.set_option("timing", 1)
+    for _ in range(max(3, args.warmup)):
+        step()
+    barrier()
+    gev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    replays = 0
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xFF)
+        gev[i][0].record(stream)
+        C = step()
+        gev[i][1].record(stream)
+        replays += h.stats()["graph_replays"]
+        del C
+    barrier()
+    g_ms = sum(a.elapsed_time(b) for a, b in gev)
+    gt = torch.tensor([g_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(gt, op=dist.ReduceOp.MAX)
+    graph_replay = {"value": 2 * total_nprod * args.steps / (float(gt.item()) / 1e3) / 1e9, "unit": UNIT,
+                    "ms_per_step": float(gt.item()) / args.steps, "segments_replayed": int(replays)}
+
     # end to end through the public API from pinned host buffers
     e2e = None
     if not args.no_e2e:
@@ -323,7 +348,7 @@ def run_ours(args):
                 "warmup": args.warmup, "ms_per_step": max_ms / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
                 "config": config_dict(args, A, world), "impl": "ours",
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "graph_replay": graph_replay,
                 "gpu_launches": int(launches), "clocks": clk.summary(),
                 "nprod": int(total_nprod), "nnz_c": int(st["nnz_c"]), "phase_ms_median": phases,
                 "step_ms": step_ms, "wall_s": t_wall,

@@ -23,7 +23,8 @@
  * Ownership: the caller owns A, B and all of C.  The library owns only its workspace
  * (grouping arrays, n_prod, global-memory hash tables), obtained from the allocator given to
  * spgemm_create (NULL -> a private stream-ordered CUDA memory pool of the handle whose
- * memory stays mapped between calls and is released by spgemm_destroy).  A's and B's structure
+ * memory stays mapped between calls and is released by spgemm_destroy).  Workspace buffers
+ * are grow-only: kept across calls (stable addresses for graph replay) until spgemm_destroy.  A's and B's structure
  * arrays are BORROWED from spgemm_symbolic until the next spgemm_symbolic/destroy: they
  * must stay alive and unchanged while spgemm_numeric may be called (structure reuse).
  *
@@ -123,7 +124,9 @@ typedef enum {
     SPGEMM_OPT_VALIDATE = 4,        /* 1 = O(nnz) input validation in spgemm_symbolic */
     SPGEMM_OPT_LANES = 5,           /* lanes per B row (power of two 1..32), 0 = auto */
     SPGEMM_OPT_WORKSPACE_BUDGET = 6,/* max bytes for global-memory hash tables */
-    SPGEMM_OPT_TIMING = 7,          /* 1 = per-group CUDA-event timing (default 1) */
+    SPGEMM_OPT_TIMING = 7,          /* 0 off; 1 (default) phase events, plus per-group kernel events
+                                       when graphs are off; 2 per-group kernel events always (disables
+                                       graph capture: events inside a graph cannot be timed) */
     SPGEMM_OPT_LONG_ROW = 8,        /* CTA-per-row groups: B rows longer than v are walked by
                                        the whole CTA (0 = auto, -1 = off) */
     SPGEMM_OPT_RANGE_HASH = 9,      /* 1 (default): rows whose column span fits the group's table
@@ -134,9 +137,13 @@ typedef enum {
                                        the global-memory fallback; 0: straight to global memory */
     SPGEMM_OPT_CLUSTER_FILL_LIMIT = 11, /* symbolic cluster table: rows with more distinct keys
                                        than v go to global memory (0 = capacity/2) */
-    SPGEMM_OPT_FLAT = 12            /* product loop: 1 load-balanced flattened (lanes share a batch
+    SPGEMM_OPT_FLAT = 12,           /* product loop: 1 load-balanced flattened (lanes share a batch
                                        of A non-zeros), 0 VW lanes per A non-zero, -1 auto (1 when
                                        the mean B row is shorter than 16) */
+    SPGEMM_OPT_GRAPHS = 13          /* 1 (default): the asynchronous segments (phase-1 group kernels
+                                       + scan, phase-2 group kernels, on their forked streams) are
+                                       captured into CUDA graphs and replayed while inputs,
+                                       workspace and group histogram are unchanged */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);
@@ -159,6 +166,7 @@ typedef struct {
     int64_t kernel_launches_symbolic, kernel_launches_numeric;
     int64_t workspace_bytes, workspace_peak_bytes;
     int64_t sym_overflow2_rows;         /* rows that overflowed the cluster table (global memory) */
+    int64_t graph_replays;              /* captured segments replayed during the last call pair */
 } spgemm_stats_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);

@@ -24,7 +24,7 @@ STATUS = {
 OPTIONS = {
     "sym_min_group": 0, "num_min_group": 1, "sym_fill_limit": 2, "streams": 3,
     "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8, "range_hash": 9,
-    "cluster": 10, "cluster_fill_limit": 11, "flat": 12,
+    "cluster": 10, "cluster_fill_limit": 11, "flat": 12, "graphs": 13,
 }
 
 # Symbols declared in include/spgemm.h (tests check the .so exports all of them).
@@ -59,7 +59,7 @@ class Stats(ctypes.Structure):
         ("setup_ms", c_float), ("symbolic_ms", c_float), ("scan_ms", c_float), ("numeric_ms", c_float),
         ("kernel_launches_symbolic", c_int64), ("kernel_launches_numeric", c_int64),
         ("workspace_bytes", c_int64), ("workspace_peak_bytes", c_int64),
-        ("sym_overflow2_rows", c_int64),
+        ("sym_overflow2_rows", c_int64), ("graph_replays", c_int64),
     ]
 
     def to_dict(self) -> dict:

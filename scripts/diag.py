@@ -26,6 +26,7 @@ def main():
     tdt = torch.float32 if a.dtype == "f32" else torch.float64
     dA = P.CsrMatrix.from_host(A, "cuda", tdt)
     h = P.Handle()
+    h.set_option("timing", 2)  # per-group kernel events (eager launches)
     for o in a.opt:
         k, v = o.split("=")
         h.set_option(k, int(v))

@@ -34,6 +34,7 @@ def run_gpu(spg, A: Csr, B: Csr, dtype, opts=None, handle=None):
     own = handle is None
     h = handle or spg.Handle()
     try:
+        h.set_option("timing", 2)
         for k, v in (opts or {}).items():
             h.set_option(k, v)
         C = h.multiply(_dev(spg, A.astype(dtype), dtype), _dev(spg, B.astype(dtype), dtype))
@@ -206,6 +207,28 @@ def test_long_row_cta_pass(spg, long_row, dtype):
                  {"long_row": long_row, "sym_min_group": 11, "num_min_group": 10}):
         got = run_gpu(spg, A, A, dtype, opts)
         assert_parity(got, ref, dtype, what=f"{opts}")
+
+
+@pytest.mark.parametrize("graphs", [0, 1])
+def test_graph_replay(spg, graphs):
+    """Repeated multiplies on one handle replay the captured phase-1/phase-2 segments."""
+    A = synth.config("mixed:economics", "int")
+    ref = oracle.spgemm(A.astype(np.float32), A.astype(np.float32), np.float32)
+    with spg.Handle() as h:
+        h.set_option("graphs", graphs)
+        dA = _dev(spg, A, np.float32)
+        for it in range(3):
+            C = h.multiply(dA, dA)
+            torch.cuda.synchronize()
+            st = h.stats()
+            assert_parity(C.numpy() + (None,), ref, np.float32, exact=True, what=f"iter {it}")
+            if graphs and it > 0:
+                assert st["graph_replays"] >= 1
+            if graphs:
+                assert st["symbolic_ms"] > 0 and st["numeric_ms"] > 0
+            else:
+                assert max(st["num_group_ms"]) > 0 and max(st["sym_group_ms"]) > 0
+            del C
 
 
 def test_serial_streams(spg):
