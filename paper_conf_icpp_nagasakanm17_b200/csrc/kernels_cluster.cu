@@ -57,6 +57,7 @@ __global__ void __launch_bounds__(1024) k_sym_cluster(SymArgs a, const int32_t* 
   extern __shared__ __align__(16) int smem[];
   __shared__ int* s_kp[CS];
   __shared__ int s_list[kLongChunk], s_lcnt;
+  __shared__ BlockFlat<int> s_bf;
   __shared__ int s_cnt, s_abort;
   cg::cluster_group cluster = cg::this_cluster();
   const int rank = (int)cluster.block_rank();
@@ -96,7 +97,7 @@ __global__ void __launch_bounds__(1024) k_sym_cluster(SymArgs a, const int32_t* 
       __syncthreads();
       if (t == 0) s_lcnt = 1;
       for_long_products<false, true, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
-                                          a.long_len, s_list, &s_lcnt, f, stop, rank, CS);
+                                          a.long_len, s_list, &s_lcnt, &s_bf, f, stop, rank, CS);
     }
     (void)mine;
     cluster.sync();
@@ -118,6 +119,7 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
   __shared__ int* s_kp[CS];
   __shared__ VT* s_vp[CS];
   __shared__ int s_list[kLongChunk], s_lcnt;
+  __shared__ BlockFlat<VT> s_bf;
   __shared__ int s_lohi[2];
   __shared__ long long s_part[CS];
   __shared__ long long ws[33];
@@ -160,7 +162,7 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
       if (t == 0) s_lcnt = 1;
       for_long_products<true, false, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
                                          static_cast<const VT*>(a.b_val), true, row, t, 1024, a.long_len, s_list,
-                                         &s_lcnt, f, NoStop{}, rank, CS);
+                                         &s_lcnt, &s_bf, f, NoStop{}, rank, CS);
     }
     cluster.sync();
     // (b) column span of the row: min/max over every slice, reduced into CTA 0
@@ -191,18 +193,35 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
     }
     cluster.sync();
     {
-      const int per = (wb - wa + 1023) / 1024;
-      const int w0 = wa + t * per, w1 = min(wb, w0 + per);
-      long long loc = 0;
-      for (int w = w0; w < w1; ++w) loc += __popc(bits[w]);
+      // prefix popcounts over this CTA's word slice [wa, wb): warp-contiguous segments read
+      // lane-interleaved (coalesced), warp scans per 32 words
+      const int lane = t & 31, wid = t >> 5;
+      const int seg = (((wb - wa) + 1023) / 1024) * 32;  // words per warp, multiple of 32
+      const int s0 = wa + wid * seg, s1 = min(wb, s0 + seg);
+      unsigned loc = 0;
+      for (int w = s0 + lane; w < s1; w += 32) loc += __popc(bits[w]);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) loc += __shfl_xor_sync(0xffffffffu, loc, o);
       long long tot;
-      long long run = Grp<1024>::excl_scan(loc, &tot, ws);
+      long long run = Grp<1024>::excl_scan(lane == 0 ? (long long)loc : 0LL, &tot, ws);
+      run = __shfl_sync(0xffffffffu, run, 0);
       if (t == 0) {
         for (int r = 0; r < CS; ++r) cluster.map_shared_rank(s_part, r)[rank] = tot;
       }
       cluster.sync();
       for (int r = 0; r < rank; ++r) run += s_part[r];
-      for (int w = w0; w < w1; ++w) { pre[w] = (unsigned)run; run += __popc(bits[w]); }
+      for (int w0 = s0; w0 < s1; w0 += 32) {
+        const int w = w0 + lane;
+        const unsigned v = w < s1 ? __popc(bits[w]) : 0u;
+        unsigned incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const unsigned y = __shfl_up_sync(0xffffffffu, incl, o);
+          if (lane >= o) incl += y;
+        }
+        if (w < s1) pre[w] = (unsigned)(run + incl - v);
+        run += __shfl_sync(0xffffffffu, incl, 31);
+      }
     }
     cluster.sync();
     const long long c0 = a.c_rpt[row];

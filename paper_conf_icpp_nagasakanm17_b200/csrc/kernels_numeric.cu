@@ -10,11 +10,13 @@
 // B200 deviation in (b)/(c): the paper's rank sort compares every entry with
 // every other (O(nnz_i^2) per row).  Here, with [lo, hi] the row's column range (a group
 // min/max over the table after accumulation):
-//   (c1) range/NB <= 4 (banded/FEM rows): entries are scattered into NB buckets of width
-//        <= 4 and rank = bucket start + #smaller keys in the bucket (the paper's comparison
-//        rank restricted to a bucket) — a prefix count when the range fits NB;
-//   (c4) wider ranges, CTA-per-row groups: same buckets, then one warp per bucket ranks its
-//        keys by shuffle comparisons (<= 32 keys) or a per-warp bitmap + popcount prefix;
+//   (c1) entries are scattered into NB buckets of width 2^shift over [lo, hi] and a thread
+//        per key ranks it as bucket start + #smaller keys in the bucket (the paper's
+//        comparison rank restricted to a bucket) — every bucket when range/NB <= 4
+//        (banded/FEM rows), buckets of <= 8 keys in CTA-per-row groups;
+//   (c4) crowded buckets of CTA-per-row groups (> 8 keys): one warp per bucket, round-robin
+//        over the warps, ranks its keys by shuffle comparisons (<= 32 keys) or a per-warp
+//        bitmap + popcount prefix;
 //   (c2) wider ranges, sub-warp row groups (<= 128 keys): bitonic sort of the slot indices;
 //   (c3) global-memory rows: bitmap over [lo, hi] + prefix popcounts.
 // Keys are distinct, so every path writes the identical, sorted row.
@@ -62,7 +64,7 @@ __device__ __forceinline__ void num_products(const NumArgs& a, bool active, int 
   if constexpr (TPR > 32) {
     if (long_len > 0)
       for_long_products<true, false, VT>(a.a_rpt, a.a_col, av, a.b_rpt, a.b_col, bv, active, row, t, TPR, long_len,
-                                         s_list, s_lcnt, f, NoStop{});
+                                         s_list, s_lcnt, bf, f, NoStop{});
   }
 }
 
@@ -126,7 +128,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
             if (long_len > 0)
               for_long_products<true, false, VT, true>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
                                                        a.b_col, static_cast<const VT*>(a.b_val), true, row, t, TPR,
-                                                       long_len, s_list, s_lcnt, f, NoStop{});
+                                                       long_len, s_list, s_lcnt, bf, f, NoStop{});
           }
           Grp<TPR>::sync();
           const int words = (int)(Rp >> 2);
@@ -269,9 +271,6 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
     if (hi >= lo) {
       const unsigned R = (unsigned)(hi - lo);
       while ((R >> shift) >= (unsigned)NB) ++shift;
-      // (c4) ranks dense buckets with a per-warp bitmap of 32*kWarpBitmapWords columns, so
-      // wide buckets cost nothing extra there while empty buckets cost a warp visit each.
-      if (TPR > 32 && shift > 2 && shift < 10) shift = 10;
       nb = (int)(R >> shift) + 1;
     }
     if (shift <= 2 || TPR > 32) {
@@ -307,77 +306,91 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
       }
       Grp<TPR>::sync();
       if (t == 0 && active && cn != n_total) atomicOr(a.err_flags, 2);
-      if (shift <= 2) {
-        // (c1) rank = bucket start + #smaller keys in the bucket (<= 4 keys per bucket)
-        if (active) {
-          for (int p = t; p < (int)n_total; p += TPR) {
-            const unsigned s = S[p];
-            const int key = Kp[s];
-            const int b = (key - lo) >> shift;
-            const int st = Bc[b], en = Bc[b + 1];
-            int r = st;
-            for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
-            if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
-          }
+      // (c1) thread per key: rank = bucket start + #smaller keys in its bucket, for buckets of at
+      // most kSparseBucket keys (every bucket when shift <= 2: width <= 4)
+      constexpr int kSparseBucket = 8;
+      if (active) {
+        for (int p = t; p < (int)n_total; p += TPR) {
+          const unsigned s = S[p];
+          const int key = Kp[s];
+          const int b = (key - lo) >> shift;
+          const int st = Bc[b], en = Bc[b + 1];
+          if (TPR > 32 && en - st > kSparseBucket) continue;  // crowded: (c4) below
+          int r = st;
+          for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
+          if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
         }
-      } else if constexpr (TPR > 32) {
-        // (c4) one warp per bucket: <= 32 keys -> rank by shuffle comparisons; denser buckets
-        // of width <= 1024 -> per-warp bitmap + popcount prefix; wider -> comparisons.
-        constexpr int MW = kWarpBitmapWords<TPR>;  // bitmap words per warp (32 per 1024 columns)
+      }
+      if constexpr (TPR > 32) {
+        // (c4) crowded buckets, one warp each: the warp scans 32 bucket counts at a time and
+        // visits only the crowded ones (sparse wide rows — graph shapes — have ~1 key per
+        // bucket and no warp work here).  <= 32 keys -> rank by shuffle comparisons; denser
+        // buckets of width <= 32 * kWarpBitmapWords -> per-warp bitmap + popcount prefix; wider
+        // -> comparisons.
+        constexpr int MW = kWarpBitmapWords<TPR>;  // bitmap words per warp
         constexpr int WPL = MW / 32;
         const int wid = t >> 5, ln = t & 31;
         unsigned* wb = wscr + wid * 2 * MW;
         unsigned* wp = wb + MW;
         const int words = (int)(((1u << shift) + 31) >> 5);
-        for (int b = wid; b < nb; b += TPR / 32) {
-          const int st = Bc[b], en = Bc[b + 1], c = en - st;  // warp-uniform
-          if (c == 0 || !active) continue;
-          const int base = lo + (b << shift);
-          if (c <= 32) {
-            const unsigned slot = ln < c ? (unsigned)S[st + ln] : 0u;
-            const int key = ln < c ? Kp[slot] : INT_MAX;
-            int r = 0;
-            for (int m = 0; m < c; ++m) r += __shfl_sync(0xffffffffu, key, m) < key;
-            if (ln < c && st + r < cn) { cc[st + r] = key; cv[st + r] = Vp[slot]; }
-          } else if (words <= MW) {
-            for (int w = ln; w < words; w += 32) wb[w] = 0u;
-            __syncwarp();
-            for (int p = st + ln; p < en; p += 32) {
-              const unsigned d = (unsigned)(Kp[S[p]] - base);
-              atomicOr(wb + (d >> 5), 1u << (d & 31));
-            }
-            __syncwarp();
-            unsigned loc[WPL], sum = 0;
+        // bucket b belongs to warp b % NW (crowded buckets are usually adjacent — the dense
+        // part of a row's column range — so a round-robin split balances them over the warps)
+        constexpr int NW = TPR / 32;
+        for (int k0 = 0; active && wid + k0 * NW < nb; k0 += 32) {
+          const int bl = wid + (k0 + ln) * NW;
+          const int cl = bl < nb ? Bc[bl + 1] - Bc[bl] : 0;
+          unsigned crowd = __ballot_sync(0xffffffffu, cl > kSparseBucket);
+          while (crowd) {
+            const int b = wid + (k0 + __ffs(crowd) - 1) * NW;
+            crowd &= crowd - 1;
+            const int st = Bc[b], en = Bc[b + 1], c = en - st;  // warp-uniform
+            const int base = lo + (b << shift);
+            if (c <= 32) {
+              const unsigned slot = ln < c ? (unsigned)S[st + ln] : 0u;
+              const int key = ln < c ? Kp[slot] : INT_MAX;
+              int r = 0;
+              for (int m = 0; m < c; ++m) r += __shfl_sync(0xffffffffu, key, m) < key;
+              if (ln < c && st + r < cn) { cc[st + r] = key; cv[st + r] = Vp[slot]; }
+            } else if (words <= MW) {
+              for (int w = ln; w < words; w += 32) wb[w] = 0u;
+              __syncwarp();
+              for (int p = st + ln; p < en; p += 32) {
+                const unsigned d = (unsigned)(Kp[S[p]] - base);
+                atomicOr(wb + (d >> 5), 1u << (d & 31));
+              }
+              __syncwarp();
+              unsigned loc[WPL], sum = 0;
 #pragma unroll
-            for (int u = 0; u < WPL; ++u) {
-              loc[u] = ln * WPL + u < words ? __popc(wb[ln * WPL + u]) : 0u;
-              sum += loc[u];
-            }
-            unsigned incl = sum;
+              for (int u = 0; u < WPL; ++u) {
+                loc[u] = ln * WPL + u < words ? __popc(wb[ln * WPL + u]) : 0u;
+                sum += loc[u];
+              }
+              unsigned incl = sum;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-              const unsigned y = __shfl_up_sync(0xffffffffu, incl, o);
-              if (ln >= o) incl += y;
-            }
-            unsigned ex = incl - sum;
+              for (int o = 1; o < 32; o <<= 1) {
+                const unsigned y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (ln >= o) incl += y;
+              }
+              unsigned ex = incl - sum;
 #pragma unroll
-            for (int u = 0; u < WPL; ++u) { wp[ln * WPL + u] = ex; ex += loc[u]; }
-            __syncwarp();
-            for (int p = st + ln; p < en; p += 32) {
-              const unsigned slot = S[p];
-              const int key = Kp[slot];
-              const unsigned d = (unsigned)(key - base);
-              const int r = st + (int)wp[d >> 5] + __popc(wb[d >> 5] & ((1u << (d & 31)) - 1u));
-              if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
-            }
-            __syncwarp();
-          } else {
-            for (int p = st + ln; p < en; p += 32) {
-              const unsigned slot = S[p];
-              const int key = Kp[slot];
-              int r = st;
-              for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
-              if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
+              for (int u = 0; u < WPL; ++u) { wp[ln * WPL + u] = ex; ex += loc[u]; }
+              __syncwarp();
+              for (int p = st + ln; p < en; p += 32) {
+                const unsigned slot = S[p];
+                const int key = Kp[slot];
+                const unsigned d = (unsigned)(key - base);
+                const int r = st + (int)wp[d >> 5] + __popc(wb[d >> 5] & ((1u << (d & 31)) - 1u));
+                if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
+              }
+              __syncwarp();
+            } else {
+              for (int p = st + ln; p < en; p += 32) {
+                const unsigned slot = S[p];
+                const int key = Kp[slot];
+                int r = st;
+                for (int q = st; q < en; ++q) r += (Kp[S[q]] < key);
+                if (r < cn) { cc[r] = key; cv[r] = Vp[slot]; }
+              }
             }
           }
         }

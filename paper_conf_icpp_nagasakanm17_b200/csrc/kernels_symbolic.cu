@@ -44,7 +44,7 @@ __device__ __forceinline__ void sym_products(const SymArgs& a, bool active, int 
   if constexpr (TPR > 32) {
     if (long_len > 0)
       for_long_products<false, STOP, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, active, row, t, TPR,
-                                          long_len, s_list, &s_lcnt, f, stop);
+                                          long_len, s_list, &s_lcnt, bf, f, stop);
   }
 }
 
@@ -180,7 +180,7 @@ __global__ __launch_bounds__(1024) void k_sym_global(SymArgs a) {
                                         a.vw_log2, f, NoStop{}, a.long_len, &s_lcnt);
       if (a.long_len > 0)
         for_long_products<false, false, int>(a.a_rpt, a.a_col, nullptr, a.b_rpt, a.b_col, nullptr, true, row, t, 1024,
-                                             a.long_len, s_list, &s_lcnt, f, NoStop{});
+                                             a.long_len, s_list, &s_lcnt, &s_bf, f, NoStop{});
     }
     const long long tot = Grp<1024>::sum(cnt, ws);
     if (t == 0) a.c_cnt[row] = tot;

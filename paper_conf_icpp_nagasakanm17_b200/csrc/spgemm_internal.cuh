@@ -410,9 +410,13 @@ __device__ __forceinline__ void products(bool flat, const int64_t* __restrict__ 
 
 // Second pass (CTA-wide, every thread of the CTA must call it): the A row is rescanned in
 // chunks of kLongChunk entries; entries whose B row is longer than long_len go to a shared
-// list, and all tpr threads stride each listed B row (unrolled by 2).  s_list: kLongChunk
-// ints, s_cnt: one int, both shared; s_cnt must be 0 before pass 1 and is set by pass 1 when
-// it defers a row (otherwise this pass returns at once).  A stopped (CHECK_STOP) thread keeps
+// list (s_list: kLongChunk ints, s_cnt: one int; s_cnt must be 0 before pass 1 and is set by
+// pass 1 when it defers a row, otherwise this pass returns at once).  The listed B rows are then
+// walked flattened: their lengths are scanned into bf->incl and every thread strides the
+// concatenated products, so a chunk with many long rows keeps all tpr threads' gathers in flight
+// instead of walking the rows one after another (R-MAT hub rows: measured 40x on cluster rows).
+// WSYNC (private-accumulator rows, where the lanes of a sub-group must hold distinct columns of
+// one B row) walks the listed rows one at a time instead.  A stopped (CHECK_STOP) thread keeps
 // hitting barriers.
 constexpr int kLongChunk = 256;
 template <bool NUM, bool CHECK_STOP, typename VT, bool WSYNC = false, typename F, typename S>
@@ -420,7 +424,8 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
                                                   const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                   const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
                                                   bool active, int row, int t, int tpr, int long_len, int* s_list,
-                                                  int* s_cnt, F&& f, S&& stop, int part = 0, int nparts = 1) {
+                                                  int* s_cnt, BlockFlat<VT>* bf, F&& f, S&& stop, int part = 0,
+                                                  int nparts = 1) {
   const long long a0 = active ? __ldg(a_rpt + row) : 0;
   const int32_t* __restrict__ ac = a_col + a0;
   __syncthreads();  // s_cnt doubles as the "some sub-group deferred a row" flag of pass 1
@@ -441,31 +446,79 @@ __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_
     }
     if (__syncthreads_count(added) == 0) continue;  // no long row in this chunk: one barrier
     const int n = *s_cnt;
-    for (int i = 0; i < n; ++i) {
-      const int j = s_list[i];
-      const int kk = __ldg(ac + j);
-      const VT av = NUM ? __ldg(a_val + a0 + j) : VT(0);
-      const long long b0 = __ldg(b_rpt + kk);
-      int len = (int)(__ldg(b_rpt + kk + 1) - b0);
-      if (CHECK_STOP && stop()) len = 0;
-      const int32_t* __restrict__ bc = opaque(b_col + b0);
-      const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
+    if constexpr (WSYNC) {
+      for (int i = 0; i < n; ++i) {
+        const int j = s_list[i];
+        const int kk = __ldg(ac + j);
+        const VT av = NUM ? __ldg(a_val + a0 + j) : VT(0);
+        const long long b0 = __ldg(b_rpt + kk);
+        int len = (int)(__ldg(b_rpt + kk + 1) - b0);
+        if (CHECK_STOP && stop()) len = 0;
+        const int32_t* __restrict__ bc = opaque(b_col + b0);
+        const VT* __restrict__ bv = NUM ? opaque(b_val + b0) : nullptr;
 #pragma unroll 1
-      for (int q = t; q < len; q += 2 * tpr) {
-        const int k0 = __ldg(bc + q);
-        const VT v0 = NUM ? __ldg(bv + q) : VT(0);
-        const bool h1 = q + tpr < len;
-        int k1 = 0;
-        VT v1 = VT(0);
-        if (h1) { k1 = __ldg(bc + q + tpr); if (NUM) v1 = __ldg(bv + q + tpr); }
-        if (CHECK_STOP && stop()) break;
-        f(k0, av * v0);
-        if (h1) {
-          if (CHECK_STOP && stop()) break;
-          f(k1, av * v1);
-        }
+        for (int q = t; q < len; q += tpr) f(__ldg(bc + q), NUM ? av * __ldg(bv + q) : VT(0));
+        __syncwarp();
       }
-      if constexpr (WSYNC) __syncwarp();
+    } else {
+      // listed rows' (start, value, length) -> shared; inclusive scan of the lengths by warps
+      const int lane = t & 31, wid = t >> 5, nw = tpr >> 5;
+      for (int i = t; i < n; i += tpr) {
+        const int j = s_list[i];
+        const int kk = __ldg(ac + j);
+        const long long b0 = __ldg(b_rpt + kk);
+        bf->b0[i] = b0;
+        bf->incl[i] = (int)(__ldg(b_rpt + kk + 1) - b0);
+        if (NUM) bf->av[i] = __ldg(a_val + a0 + j);
+      }
+      __syncthreads();
+      for (int blk = wid; blk * 32 < n; blk += nw) {
+        const int e = blk * 32 + lane;
+        int v = e < n ? bf->incl[e] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(0xffffffffu, v, o);
+          if (lane >= o) v += y;
+        }
+        if (e < n) bf->incl[e] = v;
+      }
+      __syncthreads();
+      int addv[kLongChunk / 64 + 1];  // per-thread fix-ups for its elements (n <= kLongChunk)
+#pragma unroll
+      for (int u = 0; u < kLongChunk / 64 + 1; ++u) {
+        const int e = t + u * tpr;
+        int add = 0;
+        if (e < n)
+          for (int b = 0; b < (e >> 5); ++b) add += bf->incl[b * 32 + 31];
+        addv[u] = add;
+      }
+      __syncthreads();
+#pragma unroll
+      for (int u = 0; u < kLongChunk / 64 + 1; ++u) {
+        const int e = t + u * tpr;
+        if (e < n) bf->incl[e] += addv[u];
+      }
+      __syncthreads();
+      const int P = bf->incl[n - 1];
+      int e = 0;
+      {  // first entry with incl > t (binary search), then advance monotonically with p
+        int lo = 0, hi = n - 1;
+        while (lo < hi) {
+          const int mid = (lo + hi) >> 1;
+          if (bf->incl[mid] <= t) lo = mid + 1; else hi = mid;
+        }
+        e = lo;
+      }
+#pragma unroll 1
+      for (int p = t; p < P; p += tpr) {
+        while (bf->incl[e] <= p) ++e;
+        const int start = e ? bf->incl[e - 1] : 0;
+        const long long q = bf->b0[e] + (p - start);
+        const int key = __ldg(b_col + q);
+        const VT v = NUM ? __ldg(b_val + q) : VT(0);
+        if (CHECK_STOP && stop()) break;
+        f(key, NUM ? bf->av[e] * v : VT(0));
+      }
     }
     __syncthreads();
     if (t == 0) *s_cnt = 0;

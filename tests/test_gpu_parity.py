@@ -387,3 +387,47 @@ def test_rmat_s20_sampled(spg):
         assert e - s == r_rpt[1]
         assert np.array_equal(col[s:e], r_col)
         assert np.all(np.abs(val[s:e] - r_val) <= 1e-5 * r_abs)
+
+
+def _sampled_rows_parity(C, A32, rows, rtol):
+    """Compare the listed rows of a device C with the oracle, one row at a time, copying only
+    those rows to the host (C may be tens of GB)."""
+    rpt = C.rpt.cpu().numpy()
+    for r in rows:
+        r = int(r)
+        S = oracle.row_slice(A32, r, r + 1)
+        r_rpt, r_col, r_val, r_abs = oracle.spgemm(S, A32, np.float32)
+        s, e = int(rpt[r]), int(rpt[r + 1])
+        assert e - s == r_rpt[1], f"row {r}: nnz {e - s} != {r_rpt[1]}"
+        assert np.array_equal(C.col[s:e].cpu().numpy(), r_col), f"row {r}: col differs"
+        v = C.val[s:e].cpu().numpy()
+        assert np.all(np.abs(v.astype(np.float64) - r_val) <= rtol * r_abs), f"row {r}: values"
+    return rpt
+
+
+@pytest.mark.slow
+def test_rmat_s22_sampled(spg):
+    """Config 5 at full single-GPU size: R-MAT(0.45,0.15,0.15,0.25) s22 ef16, nnz(C) > 2^31
+    (int64 rpt path), sampled rows + heaviest rows against the oracle, global invariants."""
+    A = synth.rmat(22).with_values("uniform", 7)
+    A32 = A.astype(np.float32)
+    with spg.Handle() as h:
+        dA = _dev(spg, A32, np.float32)
+        C = h.multiply(dA, dA)
+        torch.cuda.synchronize()
+        st = h.stats()
+        _, total = oracle.nprod(A32, A32)
+        assert h.nprod == total
+        assert C.nnz > 2**31 - 1  # exercises 64-bit row pointers / output offsets
+        rng = np.random.default_rng(1)
+        lens = (A.rpt[1:] - A.rpt[:-1])
+        heavy = np.argsort(lens)[-8:]
+        rows = np.concatenate([rng.integers(0, A.m, 60), heavy, [0, A.m - 1]])
+        rpt = _sampled_rows_parity(C, A32, rows, 1e-5)
+        assert rpt[0] == 0 and np.all(np.diff(rpt) >= 0) and rpt[-1] == C.nnz
+        # every output row strictly increasing: device-side check over all of C
+        d = C.col[1:].to(torch.int64) - C.col[:-1].to(torch.int64)
+        starts = torch.zeros(C.nnz, dtype=torch.bool, device=C.col.device)
+        starts[C.rpt[1:-1][C.rpt[1:-1] < C.nnz]] = True
+        assert bool(((d > 0) | starts[1:]).all())
+        assert st["nnz_c"] == C.nnz
