@@ -140,10 +140,16 @@ typedef enum {
     SPGEMM_OPT_FLAT = 12,           /* product loop: 1 load-balanced flattened (lanes share a batch
                                        of A non-zeros), 0 VW lanes per A non-zero, -1 auto (1 when
                                        the mean B row is shorter than 16) */
-    SPGEMM_OPT_GRAPHS = 13          /* 1 (default): the asynchronous segments (phase-1 group kernels
+    SPGEMM_OPT_GRAPHS = 13,         /* 1 (default): the asynchronous segments (phase-1 group kernels
                                        + scan, phase-2 group kernels, on their forked streams) are
                                        captured into CUDA graphs and replayed while inputs,
                                        workspace and group histogram are unchanged */
+    SPGEMM_OPT_RANGE_WARP = 14,     /* 1 (default): "range rows" — exact column span R_i <= 2048,
+                                       R_i <= 4 n_prod_i, n_prod_i in [RANGE_MIN_NPROD, 65536] — are
+                                       counted and computed by warp-per-row kernels over an offset
+                                       table of R_i slots; 0: Table-I groups only.
+                                       Needs RANGE_HASH; off while a MIN_GROUP is forced */
+    SPGEMM_OPT_RANGE_MIN_NPROD = 15 /* n_prod lower bound of range rows (default 256) */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

@@ -6,7 +6,7 @@ C = A * B with A, B, C in CSR (int64 rpt, int32 col, fp32/fp64 values):
 The kernels live in libspgemm.so (csrc/, C ABI in include/spgemm.h); this package only
 marshals arguments.  See DESIGN.md.
 """
-from ._lib import SpgemmError, group_bounds, load  # noqa: F401
+from ._lib import NUM_RANGE_GROUP, SYM_RANGE_GROUP, SpgemmError, group_bounds, load  # noqa: F401
 from .spgemm import CsrMatrix, Handle, spgemm  # noqa: F401
 
 __all__ = ["CsrMatrix", "Handle", "spgemm", "group_bounds", "load", "SpgemmError"]

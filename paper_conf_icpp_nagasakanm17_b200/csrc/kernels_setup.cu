@@ -133,15 +133,28 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
     }
     if (lane == src) { np = part; lo = plo; hi = phi; }
   }
-  int g = -1;
+  int g = -1, span = 0;
   if (row < m) {
     nprod[row] = np;
     if (rlohi) rlohi[row] = make_int2(lo, hi);
-    if (np == 0) c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
-    else g = group_of(np, bd);
+    if (np == 0) {
+      c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
+    } else {
+      const long long R = (long long)hi - lo + 1;
+      // range rows (kernels_range.cu): narrow exact column span, enough products for a warp
+      if (bd.range_group >= 0 && rlohi && np >= bd.range_min_np && np <= kRangeMaxNprod && R <= kRangeMaxSpan &&
+          R <= kRangeSpanPerProd * np && __ldg(b_rpt + bd.range_k) < (1LL << 31)) {
+        g = bd.range_group;
+        span = (int)R;
+      } else {
+        g = group_of(np, bd);
+      }
+    }
     grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
   }
   count_group(g >= 0, g, s_cnt);
+  span = __reduce_max_sync(0xffffffffu, span);
+  if (lane == 0 && span > 0) atomicMax(&acc->range_rmax, span);
   const unsigned long long tot = warp_sum_u64((unsigned long long)np);
   const unsigned long long mx = warp_max_u64((unsigned long long)np);
   if (lane == 0) { atomicAdd(&s_total, tot); atomicMax(&s_max, mx); }
@@ -198,6 +211,7 @@ __device__ __forceinline__ long long block_sum_ll(long long v, long long* ws) {
 // (group ids, per-group row counts and the maximum nnz_i: what the host needs at sync 2).
 __global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(long long m, const int64_t* __restrict__ x,
                                                                long long* __restrict__ tile_sums,
+                                                               const uint8_t* __restrict__ grp1,
                                                                uint8_t* __restrict__ grp2, DevAcc* __restrict__ acc,
                                                                Bounds bd) {
   __shared__ long long ws[33];
@@ -220,7 +234,7 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(long long m, cons
     if (grouping) {  // block-uniform branch
       int g = -1;
       if (i < m) {
-        if (v > 0) g = group_of(v, bd);
+        if (v > 0) g = (bd.range_group >= 0 && grp1[i] == kSymRange) ? bd.range_group : group_of(v, bd);
         grp2[i] = (uint8_t)(g < 0 ? 0xFF : g);
       }
       count_group(g >= 0, g, s_cnt);
@@ -410,22 +424,20 @@ size_t scan_workspace_bytes(long long m) {
   return (size_t)((m + kScanTile - 1) / kScanTile + 1) * sizeof(long long);
 }
 
-static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, uint8_t* grp2, DevAcc* acc, Bounds b,
-                                  long long* tile_ws, long long* total_out, int* nlaunch) {
+static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const uint8_t* grp1, uint8_t* grp2,
+                                  DevAcc* acc, Bounds b, long long* tile_ws, long long* total_out, int* nlaunch) {
   if (m == 0) return cudaSuccess;
   const long long ntiles = (m + kScanTile - 1) / kScanTile;
-  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, grp2, acc, b);
+  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, grp1, grp2, acc, b);
   k_scan_tiles<<<1, 1024, 0, s>>>(ntiles, tile_ws);
   k_scan_down<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, total_out);
   if (nlaunch) *nlaunch += 3;
   return cudaGetLastError();
 }
 
-cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const int64_t* nprod,
-                                  const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
-                                  long long* tile_ws, int* nlaunch) {
-  (void)nprod; (void)a_rpt;
-  return scan_inclusive(s, m, c_rpt + 1, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
+cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const uint8_t* grp1,
+                                  uint8_t* grp2, DevAcc* acc, Bounds b, long long* tile_ws, int* nlaunch) {
+  return scan_inclusive(s, m, c_rpt + 1, grp1, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
 }
 
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
@@ -443,7 +455,8 @@ cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, 
     const long long rpb = kSetupThreads / 32;
     k_nprod_only<<<(unsigned)((m + rpb - 1) / rpb), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod_scan + 1);
     Bounds none{};
-    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
+    none.range_group = -1;
+    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
     if (e != cudaSuccess) return e;
   }
   k_splits<<<(nparts + 1 + 255) / 256, 256, 0, s>>>(m, nprod_scan, nparts, splits_dev);

@@ -82,6 +82,8 @@ struct spgemm_ctx {
   int use_cluster = 1;   // 0: rows beyond one CTA go straight to global memory (ablation)
   int flat = -1;         // load-balanced flattened product loop: -1 auto (mean B row < 16), 0, 1
   int timing = 1;
+  int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
+  long long range_min_np = kRangeMinNprodDefault;
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
   int state = 0;
@@ -91,7 +93,9 @@ struct spgemm_ctx {
   const int32_t *a_col = nullptr, *b_col = nullptr;
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
-  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi, num_slab, num_slab_c;
+  Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi, num_slab, num_slab_c,
+      rbits;
+  bool range_num = false;  // numeric range rows on for the last symbolic call (bitmap allocated, B sorted)
   GraphCache gsym, gnum;  // captured segments (see run_graph)
   int use_graphs = 1;
   bool perm2_ready = false;
@@ -170,7 +174,7 @@ void release_state(spgemm_handle_t h) {
 
 void free_all(spgemm_handle_t h) {
   Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow,
-                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c};
+                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits};
   for (Buf* b : all) buf_free(h, *b);
   release_state(h);
 }
@@ -237,19 +241,31 @@ spgemm_status_t run_graph(spgemm_handle_t h, GraphCache& gc, const std::vector<l
     if (s_ != SPGEMM_OK) return s_;                                \
   } while (0)
 
-Bounds sym_bounds(int min_group) {
+// Range rows (kernels_range.cu) need the column spans (range hash on) and are not used when a
+// minimum group is forced (the forced-path tests pin every hash-table group).
+bool sym_range_on(spgemm_handle_t h) { return h->range_warp && h->range_hash && h->sym_min_group < 0; }
+
+Bounds sym_bounds(spgemm_handle_t h) {
   Bounds b{};
   for (int i = 0; i < kNumSymBounds; ++i) b.upper[i] = kSymGroups[i].upper;
   b.nbounds = kNumSymBounds;
-  b.min_group = min_group;
+  b.min_group = h->sym_min_group;
+  b.range_group = sym_range_on(h) ? kSymRange : -1;
+  b.range_min_np = h->range_min_np;
+  b.range_k = h->k;
   return b;
 }
 
-Bounds num_bounds(int min_group) {
+// Numeric range rows: the phase-1 range rows, when every B row is strictly increasing (plain
+// read-modify-write accumulation), the pattern bitmap fits the workspace budget and no numeric
+// group is forced (decided at sync 1: h->range_num).
+Bounds num_bounds(spgemm_handle_t h) {
   Bounds b{};
   for (int i = 0; i < kNumNumBounds; ++i) b.upper[i] = kNumGroups[i].upper;
   b.nbounds = kNumNumBounds;
-  b.min_group = min_group;
+  b.min_group = h->num_min_group;
+  b.range_group = h->range_num ? kNumRange : -1;
+  b.range_min_np = 0;
   return b;
 }
 
@@ -482,6 +498,10 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_CLUSTER_FILL_LIMIT:
       if (v < 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "CLUSTER_FILL_LIMIT < 0");
       h->cluster_fill = (int)std::min<int64_t>(v, 1 << 30); break;
+    case SPGEMM_OPT_RANGE_WARP: h->range_warp = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANGE_MIN_NPROD:
+      if (v < 1 || v > kRangeMaxNprod) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_MIN_NPROD out of range");
+      h->range_min_np = v; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -546,7 +566,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
     int nl = 0;
     CK(launch_nprod_group(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, static_cast<int2*>(h->bmm.p),
                           static_cast<int64_t*>(h->nprod.p), static_cast<int2*>(h->rlohi.p),
-                          static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h->sym_min_group), &nl));
+                          static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h), &nl));
     launches += nl;
   }
   CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
@@ -596,18 +616,31 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.slab_T = slab_T;
   sa.nprod = static_cast<int64_t*>(h->nprod.p);
   sa.n = n;
+  // range rows: pattern bitmap (symbolic -> numeric gather), rwcap words per row of the group
+  const long long n_range = (long long)h->snap1.sym_rows[kSymRange];
+  h->range_num = false;
+  if (n_range > 0) {
+    sa.rwcap = range_wcap(h->snap1.range_rmax);
+    const long long bytes = n_range * sa.rwcap * 4;  // <= 256 B per range row
+    if (bytes <= h->ws_budget) {
+      ALLOC(h->rbits, (size_t)bytes);
+      sa.rbits = static_cast<unsigned*>(h->rbits.p);
+      h->range_num = h->snap1.b_unsorted == 0 && h->num_min_group < 0;
+    }
+  }
   const int32_t* perm1 = static_cast<const int32_t*>(h->perm1.p);
   // segment 2 of phase 1 (scatter, per-group kernels on forked streams, scan): captured once per
   // (inputs, workspace, group histogram, options) and replayed
   std::vector<long long> topo = {1, m, k, n, glob_grid, slab_T, h->vw_log2, sa.long_len, sa.flat, sa.fill_limit,
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
-                                 h->range_hash, (long long)group_events(h)};
+                                 h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
+                                 h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
                                        (long long)h->slab_sym.p, (long long)h->overflow.p, (long long)h->overflow2.p,
                                        (long long)h->grp2.p, (long long)h->rlohi.p, (long long)h->nprod.p,
-                                       (long long)h->tiles.p, (long long)h->grp1.p};
+                                       (long long)h->tiles.p, (long long)h->grp1.p, (long long)h->rbits.p};
   int seg_launches = 0;
   const bool ge = group_events(h);
   h->gtimed_phases = ge && h->timing;
@@ -652,6 +685,17 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       if (ge) CK(cudaEventRecord(h->gstop[0][g], s));
       h->gtimed[0][g] = ge;
     }
+    if (h->snap1.sym_rows[kSymRange] > 0) {  // range rows: warp-per-row offset tables
+      cudaStream_t s = group_stream(h, kSymRange);
+      if (ge) CK(cudaEventRecord(h->gstart[0][kSymRange], s));
+      SymArgs ra = sa;
+      ra.rows = perm1 + off1.off[kSymRange];
+      ra.nrows = (long long)h->snap1.sym_rows[kSymRange];
+      CK(launch_symbolic_range(s, ra, h->snap1.range_rmax, h->num_sms));
+      ++launches;
+      if (ge) CK(cudaEventRecord(h->gstop[0][kSymRange], s));
+      h->gtimed[0][kSymRange] = ge;
+    }
     if (n_opt == 0 && n_glob > 0) {  // forced global group only
       cudaStream_t s = group_stream(h, kSymGlobal);
       if (ge) CK(cudaEventRecord(h->gstart[0][kSymGlobal], s));
@@ -669,8 +713,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
 
     // (4) rpt_C = prefix sum, fused with (6) grouping by nnz_i
     int nl = 0;
-    CK(launch_scan_and_group(h->stream, m, c_rpt, static_cast<int64_t*>(h->nprod.p), a_rpt,
-                             static_cast<uint8_t*>(h->grp2.p), dacc, num_bounds(h->num_min_group),
+    CK(launch_scan_and_group(h->stream, m, c_rpt, static_cast<const uint8_t*>(h->grp1.p),
+                             static_cast<uint8_t*>(h->grp2.p), dacc, num_bounds(h),
                              static_cast<long long*>(h->tiles.p), &nl));
     launches += nl;
     
@@ -747,6 +791,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const bool fp64 = dt == SPGEMM_F64;
     const long long vs = fp64 ? 8 : 4;
     const Offsets off2 = offsets_of(h->snap2.num_rows, kNumNumGroups);
+    const Offsets off1 = offsets_of(h->snap1.sym_rows, kNumSymGroups);
     DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
     NumArgs na{};
     na.a_rpt = h->a_rpt; na.a_col = h->a_col; na.a_val = a_val;
@@ -788,12 +833,14 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // phase 2 (per-group kernels on forked streams): captured once per key and replayed (e.g.
     // numeric re-runs with new values of the same structure, or repeated multiplies)
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, h->vw_log2, na.long_len, na.flat,
-                                   na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h)};
+                                   na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
+                                   h->snap1.range_rmax};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
                                          (long long)h->b_rpt, (long long)h->b_col, (long long)perm2, (long long)h->acc.p,
-                                         (long long)h->rlohi.p, (long long)h->num_slab.p, (long long)h->num_slab_c.p};
+                                         (long long)h->rlohi.p, (long long)h->num_slab.p, (long long)h->num_slab_c.p,
+                                         (long long)h->rbits.p, (long long)h->perm1.p};
     const bool ge = group_events(h);
     auto enqueue = [&]() -> spgemm_status_t {
       CK(fork(h));
@@ -807,6 +854,14 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
         ga.nrows = rows;
         if (g == kNumGlobal) {
           CK(launch_numeric_global(st, fp64, ga, glob_grid));
+        } else if (g == kNumRange) {
+          // the symbolic range rows in their phase-1 order (the bitmap's row index)
+          NumArgs ra = ga;
+          ra.rows = static_cast<const int32_t*>(h->perm1.p) + off1.off[kSymRange];
+          ra.nrows = (long long)h->snap1.sym_rows[kSymRange];
+          ra.rbits = static_cast<const unsigned*>(h->rbits.p);
+          ra.rwcap = range_wcap(h->snap1.range_rmax);
+          CK(launch_numeric_range(st, fp64, ra, h->snap1.range_rmax, h->num_sms));
         } else if (g >= kNumCluster && g < kNumCluster + 3) {
           const int c = g - kNumCluster;
           long long before = 0;

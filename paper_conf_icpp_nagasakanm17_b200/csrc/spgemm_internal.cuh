@@ -50,7 +50,8 @@ constexpr GroupSpec kSymGroups[] = {
 constexpr int kNumSymBounds = 10;   // groups 0..9 have an upper bound
 constexpr int kSymOptimistic = 10;
 constexpr int kSymGlobal = 11;
-constexpr int kNumSymGroups = 12;   // including global
+constexpr int kSymRange = 12;       // range rows: warp-per-row offset table (kernels_range.cu)
+constexpr int kNumSymGroups = 13;   // including global and range
 
 // Phase 2 (numeric), key = nnz_i.  Same bounds for fp32 and fp64 (fp64 sizes the smem).
 // Groups 10-12 = cluster-per-row (DSMEM of 2/4/8 CTAs, kernels_cluster.cu; load factor up to 3/4
@@ -70,7 +71,18 @@ constexpr GroupSpec kNumGroups[] = {
 constexpr int kNumNumBounds = 13;
 constexpr int kNumCluster = 10;  // groups 10, 11, 12: clusters of 2, 4, 8 CTAs
 constexpr int kNumGlobal = 13;
-constexpr int kNumNumGroups = 14;
+constexpr int kNumRange = 14;       // range rows (kernels_range.cu)
+constexpr int kNumNumGroups = 15;
+
+// Range rows (kernels_range.cu): column span R_i <= kRangeMaxSpan and
+// R_i <= kRangeSpanPerProd * n_prod_i, n_prod_i in [range_min_np, kRangeMaxNprod] (one warp
+// per row).  Per-CTA shared-memory budget of the per-warp tables (the rest of the SM's 256 KB
+// stays L1 for the B rows the CTA's neighbouring rows share).
+constexpr int kRangeMaxSpan = 2048;
+constexpr int kRangeSpanPerProd = 4;
+constexpr long long kRangeMaxNprod = 1 << 16;
+constexpr long long kRangeMinNprodDefault = 256;
+constexpr long long kRangeSmemBudget = 96 * 1024;
 
 // Numeric per-row shared-memory layout: vals[T] | keys[T] | bucket[NB+1] | sidx[upper] ,
 // NB = T/2 (T/8 for the largest table) buckets for the bucket-rank sort.
@@ -95,12 +107,16 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   int err_flags;  // bit0 invalid input, bit1 numeric row count mismatch
   int b_unsorted;  // some B row is not strictly increasing (disables private accumulators)
   int cursor[2][kMaxGroups];
+  int range_rmax;  // max column span R_i over the range rows (sizes the per-warp tables)
 };
 
 struct Bounds {  // group bounds passed by value
   long long upper[kMaxGroups];
   int nbounds;     // groups 0..nbounds-1 bounded; key > last bound -> group nbounds
   int min_group;   // -1 or forced minimum group
+  int range_group;  // -1, or the group id of range rows (kSymRange / kNumRange)
+  long long range_min_np;  // phase 1: n_prod lower bound of range rows
+  long long range_k;       // phase 1: rows of B (range rows need rpt_B[k] < 2^31: 32-bit offsets)
 };
 
 struct Offsets {
@@ -679,6 +695,7 @@ struct SymArgs {
   const int* dev_count;    // extra rows from overflow list (device count), may be null
   const int32_t* overflow2_rows;  // global kernel: rows that overflowed the cluster table
   const int* dev_count2;
+  unsigned* rbits; long long rwcap;  // range rows: pattern bitmap, rwcap words per row of the group
 };
 
 struct NumArgs {
@@ -694,6 +711,7 @@ struct NumArgs {
   int* err_flags;
   // global fallback
   void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;
+  const unsigned* rbits; long long rwcap;  // range rows: symbolic pattern bitmap (same row order)
 };
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
@@ -704,8 +722,8 @@ cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1,
                                const int64_t* nprod, const int64_t* a_rpt, const int64_t* c_rpt, DevAcc* acc);
 cudaError_t launch_group_scatter(cudaStream_t s, long long m, const uint8_t* grp, Offsets off,
                                  int* cursor, int32_t* perm);
-cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const int64_t* nprod,
-                                  const int64_t* a_rpt, uint8_t* grp2, DevAcc* acc, Bounds b,
+cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const uint8_t* grp1,
+                                  uint8_t* grp2, DevAcc* acc, Bounds b,
                                   long long* tile_ws, int* nlaunch);
 size_t scan_workspace_bytes(long long m);
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
@@ -721,6 +739,11 @@ cudaError_t launch_numeric_global(cudaStream_t s, bool fp64, const NumArgs& a, i
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows);
 cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);
+cudaError_t launch_symbolic_range(cudaStream_t s, const SymArgs& a, int rmax, int num_sms);
+cudaError_t launch_numeric_range(cudaStream_t s, bool fp64, const NumArgs& a, int rmax, int num_sms);
+int range_warps(long long per_warp);
+int range_rcap(long long rmax);
+int range_wcap(long long rmax);
 int cluster_capacity_sym();
 int cluster_capacity_num();
 

@@ -332,10 +332,85 @@ def test_structure_reuse_and_torch_allocator(spg):
         assert st["workspace_peak_bytes"] > 0
 
 
+# ------------------------------------------------------------------ range rows (warp-per-row)
+
+RANGE_CASES = ["cant", "mixed:protein", "mixed:accelerator", "mixed:circuit"]
+
+
+@pytest.mark.parametrize("name", RANGE_CASES)
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_range_rows(spg, name, dtype):
+    """Every row that qualifies (min n_prod lowered to 1) through the warp-per-row kernels."""
+    A = synth.config(name)
+    got = check(spg, A, A, dtype, opts={"range_min_nprod": 1}, what=f"{name} range rows")
+    st = got[3]
+    assert st["sym_rows"][spg.SYM_RANGE_GROUP] > 0
+    assert st["num_rows"][spg.NUM_RANGE_GROUP] == st["sym_rows"][spg.SYM_RANGE_GROUP]
+
+
+def test_range_rows_int_exact_and_deterministic(spg):
+    A = synth.config("cant", "int")
+    got = check(spg, A, A, np.float32, exact=True, what="cant int range")
+    assert got[3]["num_rows"][spg.NUM_RANGE_GROUP] == A.m  # every cant row is a range row
+    U = synth.config("cant")
+    a = run_gpu(spg, U, U, np.float32)
+    b = run_gpu(spg, U, U, np.float32)
+    assert np.array_equal(a[2], b[2])  # plain read-modify-write accumulation: same bits every run
+
+
+def test_range_rows_off_matches(spg):
+    A = _banded_small()
+    ref = oracle.spgemm(A, A, np.float64)
+    on = run_gpu(spg, A, A, np.float64)
+    off = run_gpu(spg, A, A, np.float64, {"range_warp": 0})
+    assert on[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0 and off[3]["sym_rows"][spg.SYM_RANGE_GROUP] == 0
+    assert_parity(on, ref, np.float64, what="range on")
+    assert_parity(off, ref, np.float64, what="range off")
+
+
+def test_range_rows_unsorted_b(spg):
+    """B rows not strictly increasing: symbolic range rows stay, numeric takes the hash groups."""
+    A = _banded_small()
+    rng = np.random.default_rng(3)
+    col = A.col.copy()
+    for i in range(0, A.m, 7):  # reverse some rows
+        s, e = A.rpt[i], A.rpt[i + 1]
+        col[s:e] = col[s:e][::-1]
+    B = Csr(A.m, A.n, A.rpt.copy(), col, A.val.copy(), name="banded_unsorted")
+    got = check(spg, A, B, np.float64, what="unsorted B")
+    assert got[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0 and got[3]["num_rows"][spg.NUM_RANGE_GROUP] == 0
+
+
+def test_range_rows_ragged(spg):
+    """Spans that are not multiples of 16/32, rows with a single A entry, empty rows, R = 1."""
+    rng = np.random.default_rng(11)
+    m = 3000
+    rows, cols = [], []
+    for i in range(m):
+        if i % 97 == 0:
+            continue  # empty row
+        w = int(rng.integers(0, 40))
+        L = int(rng.integers(1, 2 * w + 2))
+        c = np.unique(np.clip(i + rng.integers(-w, w + 1, L), 0, m - 1))
+        rows += [i] * len(c)
+        cols += c.tolist()
+    A = from_coo(m, m, np.array(rows), np.array(cols), name="ragged").with_values("uniform", 12)
+    for dtype in (np.float32, np.float64):
+        got = check(spg, A, A, dtype, opts={"range_min_nprod": 1}, what="ragged range")
+        assert got[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0
+
+
 # ------------------------------------------------------------------ intermediate steps
 
+def _block_diag(X: Csr, Y: Csr, name: str) -> Csr:
+    rpt = np.concatenate([X.rpt[:-1] - X.rpt[0], Y.rpt - Y.rpt[0] + X.nnz]).astype(np.int64)
+    col = np.concatenate([X.col, Y.col + X.n]).astype(np.int32)
+    val = np.concatenate([X.val, Y.val])
+    return Csr(X.m + Y.m, X.n + Y.n, rpt, col, val, name=name)
+
+
 def test_nprod_and_grouping(spg):
-    A = _mixed_small()
+    A = _block_diag(_mixed_small(), _banded_small(), "graph+banded")  # hash-group and range rows
     nprod_ref, total = oracle.nprod(A, A)
     ref_rpt = oracle.symbolic(A, A)
     with spg.Handle() as h:
@@ -344,9 +419,18 @@ def test_nprod_and_grouping(spg):
         nprod, perm, off = h.grouping(1)
         nprod2, perm2, off2 = h.grouping(2)
     assert np.array_equal(nprod, nprod_ref) and h.nprod == total
+    # range rows (kernels_range.cu): exact column span R_i of row i of C, from the oracle's C
+    r_rpt, r_col, _, _ = oracle.spgemm(A, A, np.float32)
+    lens = np.diff(r_rpt)
+    span = np.zeros(A.m, dtype=np.int64)
+    nz = lens > 0
+    span[nz] = r_col[r_rpt[1:][nz] - 1].astype(np.int64) - r_col[r_rpt[:-1][nz]] + 1
+    is_range = (nprod_ref >= 256) & (nprod_ref <= 65536) & (span <= 2048) & (span <= 4 * nprod_ref)
+    assert is_range.any() and (~is_range & (nprod_ref > 0)).any()  # both kinds present
     for ph, (p, o, keys) in ((1, (perm, off, nprod_ref)), (2, (perm2, off2, np.diff(ref_rpt)))):
         upper = spg.group_bounds(ph)
         want = oracle.bin_of(keys, upper)
+        want[is_range] = spg.SYM_RANGE_GROUP if ph == 1 else spg.NUM_RANGE_GROUP
         nonempty = np.flatnonzero(want >= 0)
         assert o[-1] == len(nonempty)
         assert np.array_equal(np.sort(p[:o[-1]]), nonempty)       # a permutation of grouped rows
