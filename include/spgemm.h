@@ -147,8 +147,12 @@ typedef enum {
     SPGEMM_OPT_RANGE_WARP = 14,     /* 1 (default): "range rows" — exact column span R_i <= 2048,
                                        R_i <= 4 n_prod_i, n_prod_i in [RANGE_MIN_NPROD, 65536] — are
                                        counted and computed by warp-per-row kernels over an offset
-                                       table of R_i slots; 0: Table-I groups only.
-                                       Needs RANGE_HASH; off while a MIN_GROUP is forced */
+                                       table of R_i slots; the count is a union of
+                                       B-row bitmaps when every range row has R_i <= 1024 (and the
+                                       bitmaps fit half the workspace budget), else one flag store
+                                       per product.  2: range rows, flag stores always (ablation).
+                                       0: Table-I groups only.  Needs RANGE_HASH; off while a
+                                       MIN_GROUP is forced */
     SPGEMM_OPT_RANGE_MIN_NPROD = 15 /* n_prod lower bound of range rows (default 256) */
 } spgemm_option_t;
 

@@ -32,56 +32,73 @@ __device__ __forceinline__ void count_group(bool valid, int g, int* s_cnt) {
   if (valid && lane == __ffs(peers) - 1) atomicAdd(&s_cnt[g], __popc(peers));
 }
 
-// Column range of every B row: bmm[k] = {min col, max col} ({INT_MAX, -1} if empty).  One
-// row per thread; rows longer than kLongA entries are reduced by the whole warp.
-constexpr int kLongA = 16;
+// Lanes per row of the setup kernels: power of two ~ mean row length / 4 in [1, 32], computed
+// on the device from rpt[0] and rpt[rows] (CTA-uniform); rows longer than kLongPerLane * G entries
+// go to the whole warp (power-law hub rows).
+constexpr int kLongPerLane = 16;
+__device__ __forceinline__ int setup_glog(const int64_t* __restrict__ rpt, long long rows) {
+  const long long nnz = __ldg(rpt + rows) - __ldg(rpt);
+  const long long avg = rows > 0 ? nnz / rows : 0;
+  int g = 0;
+  while (g < 5 && (4LL << g) * 2 <= avg) ++g;  // 2^g <= avg / 4
+  return g;
+}
+
+// Column range of every B row: bmm[k] = {min col, max col} ({INT_MAX, -1} if empty), and the
+// "some B row is not strictly increasing" flag.  G lanes per row (grid-stride over row blocks).
 __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, const int64_t* __restrict__ b_rpt,
                                                                const int32_t* __restrict__ b_col,
                                                                int2* __restrict__ bmm, int* __restrict__ unsorted) {
-  const int lane = threadIdx.x & 31;
-  const long long row = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
-  long long b0 = 0, b1 = 0;
-  if (row < k) { b0 = b_rpt[row]; b1 = b_rpt[row + 1]; }
-  const bool is_long = b1 - b0 > kLongA;
-  int mn = INT_MAX, mx = -1;
-  bool bad = false;  // some B row is not strictly increasing (duplicates or unsorted)
-  if (!is_long) {
-    int prev = -1;
-    for (long long j = b0; j < b1; ++j) {
-      const int c = __ldg(b_col + j);
-      mn = min(mn, c); mx = max(mx, c);
-      bad |= c <= prev;
-      prev = c;
+  const int glog = setup_glog(b_rpt, k);
+  const int G = 1 << glog, lane = threadIdx.x & 31, gl = lane & (G - 1);
+  const int rpc = kSetupThreads >> glog;
+  bool bad = false;
+  for (long long blk = (long long)blockIdx.x * rpc; blk < k; blk += (long long)gridDim.x * rpc) {
+    const long long row = blk + (threadIdx.x >> glog);
+    long long b0 = 0, b1 = 0;
+    if (row < k) { b0 = __ldg(b_rpt + row); b1 = __ldg(b_rpt + row + 1); }
+    const bool is_long = b1 - b0 > (long long)kLongPerLane * G;
+    int mn = INT_MAX, mx = -1;
+    if (!is_long) {
+      for (long long j = b0 + gl; j < b1; j += G) {
+        const int c = __ldg(b_col + j);
+        mn = min(mn, c); mx = max(mx, c);
+        if (j > b0) bad |= c <= __ldg(b_col + j - 1);
+      }
     }
-  }
-  unsigned longs = __ballot_sync(0xffffffffu, is_long);
-  while (longs) {
-    const int src = __ffs(longs) - 1;
-    longs &= longs - 1;
-    const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
-    int pmn = INT_MAX, pmx = -1;
-    bool pbad = false;
-    for (long long j = s0 + lane; j < s1; j += 32) {
-      const int c = __ldg(b_col + j);
-      pmn = min(pmn, c); pmx = max(pmx, c);
-      if (j > s0) pbad |= c <= __ldg(b_col + j - 1);
+    for (int o = G >> 1; o > 0; o >>= 1) {
+      mn = min(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+      mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
     }
+    unsigned longs = __ballot_sync(0xffffffffu, is_long && gl == 0);
+    while (longs) {
+      const int src = __ffs(longs) - 1;
+      longs &= longs - 1;
+      const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
+      int pmn = INT_MAX, pmx = -1;
+      bool pbad = false;
+      for (long long j = s0 + lane; j < s1; j += 32) {
+        const int c = __ldg(b_col + j);
+        pmn = min(pmn, c); pmx = max(pmx, c);
+        if (j > s0) pbad |= c <= __ldg(b_col + j - 1);
+      }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
-      pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
+      for (int o = 16; o > 0; o >>= 1) {
+        pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
+        pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
+      }
+      bad |= __any_sync(0xffffffffu, pbad) && lane == src;
+      if (lane == src) { mn = pmn; mx = pmx; }
     }
-    bad |= __any_sync(0xffffffffu, pbad) && lane == src;
-    if (lane == src) { mn = pmn; mx = pmx; }
+    if (row < k && gl == 0) bmm[row] = make_int2(mn, mx);
   }
-  if (row < k) bmm[row] = make_int2(mn, mx);
   if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(unsorted, 1);
 }
 
-// One row per thread; rows longer than kLongA entries are summed by the whole warp
-// (coalesced), so power-law rows do not serialise a warp behind one thread.  Also the column
-// span [lo_i, hi_i] of row i of C (min/max over its A entries of the B-row ranges): exact,
-// since every B column appears in C (kept structurally).
+// n_prod of every row (Alg. 2) with G lanes per row; also the column span [lo_i, hi_i] of row i
+// of C (min/max over its A entries of the B-row ranges): exact, since every B column appears in
+// C (kept structurally); the group id (Table I bounds, or the range-row group) and the per-group
+// histogram (CTA-aggregated before the global atomics).
 __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
     long long m, const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
     const int64_t* __restrict__ b_rpt, const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
@@ -92,77 +109,95 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
   if (threadIdx.x < kMaxGroups) s_cnt[threadIdx.x] = 0;
   if (threadIdx.x == 0) { s_total = 0; s_max = 0; }
   __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const long long row = (long long)blockIdx.x * kSetupThreads + threadIdx.x;
-  long long a0 = 0, a1 = 0;
-  if (row < m) { a0 = a_rpt[row]; a1 = a_rpt[row + 1]; }
-  const bool is_long = a1 - a0 > kLongA;
-  // Alg. 2: n_prod += rpt_B[col_A[j]+1] - rpt_B[col_A[j]], j in [rpt_A[i], rpt_A[i+1])
-  long long np = 0;
-  int lo = INT_MAX, hi = -1;
-  if (!is_long) {  // <= kLongA entries: issue the col_A loads, then the rpt_B gathers, 4 at a time
-    for (long long j = a0; j < a1; j += 4) {
-      int kk[4];
+  const int glog = setup_glog(a_rpt, m);
+  const int G = 1 << glog, lane = threadIdx.x & 31, gl = lane & (G - 1);
+  const int rpc = kSetupThreads >> glog;
+  const bool b_ok = bd.range_group >= 0 && __ldg(b_rpt + bd.range_k) < (1LL << 31);
+  unsigned long long tot = 0, mxnp = 0;
+  int span_max = 0;
+  for (long long blk = (long long)blockIdx.x * rpc; blk < m; blk += (long long)gridDim.x * rpc) {
+    const long long row = blk + (threadIdx.x >> glog);
+    long long a0 = 0, a1 = 0;
+    if (row < m) { a0 = __ldg(a_rpt + row); a1 = __ldg(a_rpt + row + 1); }
+    const bool is_long = a1 - a0 > (long long)kLongPerLane * G;
+    // Alg. 2: n_prod += rpt_B[col_A[j]+1] - rpt_B[col_A[j]], j in [rpt_A[i], rpt_A[i+1])
+    long long np = 0;
+    int lo = INT_MAX, hi = -1;
+    if (!is_long) {  // col_A loads first, then the rpt_B / span gathers, 4 entries at a time
+      for (long long j = a0 + gl; j < a1; j += 4 * G) {
+        int kk[4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) kk[u] = j + u < a1 ? __ldg(a_col + j + u) : -1;
+        for (int u = 0; u < 4; ++u) kk[u] = j + u * G < a1 ? __ldg(a_col + j + u * G) : -1;
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
-        if (kk[u] >= 0) {
-          np += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
-          if (bmm) { const int2 r = __ldg(bmm + kk[u]); lo = min(lo, r.x); hi = max(hi, r.y); }
-        }
-    }
-  }
-  unsigned longs = __ballot_sync(0xffffffffu, is_long);
-  while (longs) {
-    const int src = __ffs(longs) - 1;
-    longs &= longs - 1;
-    const long long s0 = __shfl_sync(0xffffffffu, a0, src), s1 = __shfl_sync(0xffffffffu, a1, src);
-    long long part = 0;
-    int plo = INT_MAX, phi = -1;
-    for (long long j = s0 + lane; j < s1; j += 32) {
-      const int kk = __ldg(a_col + j);
-      part += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
-      if (bmm) { const int2 r = __ldg(bmm + kk); plo = min(plo, r.x); phi = max(phi, r.y); }
-    }
-    part = (long long)warp_sum_u64((unsigned long long)part);
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      plo = min(plo, __shfl_xor_sync(0xffffffffu, plo, o));
-      phi = max(phi, __shfl_xor_sync(0xffffffffu, phi, o));
-    }
-    if (lane == src) { np = part; lo = plo; hi = phi; }
-  }
-  int g = -1, span = 0;
-  if (row < m) {
-    nprod[row] = np;
-    if (rlohi) rlohi[row] = make_int2(lo, hi);
-    if (np == 0) {
-      c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
-    } else {
-      const long long R = (long long)hi - lo + 1;
-      // range rows (kernels_range.cu): narrow exact column span, enough products for a warp
-      if (bd.range_group >= 0 && rlohi && np >= bd.range_min_np && np <= kRangeMaxNprod && R <= kRangeMaxSpan &&
-          R <= kRangeSpanPerProd * np && __ldg(b_rpt + bd.range_k) < (1LL << 31)) {
-        g = bd.range_group;
-        span = (int)R;
-      } else {
-        g = group_of(np, bd);
+        for (int u = 0; u < 4; ++u)
+          if (kk[u] >= 0) {
+            np += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+            if (bmm) { const int2 r = __ldg(bmm + kk[u]); lo = min(lo, r.x); hi = max(hi, r.y); }
+          }
       }
     }
-    grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
+    for (int o = G >> 1; o > 0; o >>= 1) {
+      np += __shfl_xor_sync(0xffffffffu, np, o);
+      lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+      hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+    }
+    unsigned longs = __ballot_sync(0xffffffffu, is_long && gl == 0);
+    while (longs) {
+      const int src = __ffs(longs) - 1;
+      longs &= longs - 1;
+      const long long s0 = __shfl_sync(0xffffffffu, a0, src), s1 = __shfl_sync(0xffffffffu, a1, src);
+      long long part = 0;
+      int plo = INT_MAX, phi = -1;
+      for (long long j = s0 + lane; j < s1; j += 32) {
+        const int kk = __ldg(a_col + j);
+        part += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
+        if (bmm) { const int2 r = __ldg(bmm + kk); plo = min(plo, r.x); phi = max(phi, r.y); }
+      }
+      part = (long long)warp_sum_u64((unsigned long long)part);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        plo = min(plo, __shfl_xor_sync(0xffffffffu, plo, o));
+        phi = max(phi, __shfl_xor_sync(0xffffffffu, phi, o));
+      }
+      if (lane == src) { np = part; lo = plo; hi = phi; }
+    }
+    const bool lead = row < m && gl == 0;
+    int g = -1;
+    if (lead) {
+      nprod[row] = np;
+      if (rlohi) rlohi[row] = make_int2(lo, hi);
+      if (np == 0) {
+        c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
+      } else {
+        const long long R = (long long)hi - lo + 1;
+        // range rows (kernels_range.cu): narrow exact column span, enough products for a warp
+        if (b_ok && rlohi && np >= bd.range_min_np && np <= kRangeMaxNprod && R <= kRangeMaxSpan &&
+            R <= kRangeSpanPerProd * np) {
+          g = bd.range_group;
+          span_max = max(span_max, (int)R);
+        } else {
+          g = group_of(np, bd);
+        }
+      }
+      grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
+      tot += (unsigned long long)np;
+      mxnp = max(mxnp, (unsigned long long)np);
+    }
+    count_group(g >= 0, g, s_cnt);
   }
-  count_group(g >= 0, g, s_cnt);
-  span = __reduce_max_sync(0xffffffffu, span);
-  if (lane == 0 && span > 0) atomicMax(&acc->range_rmax, span);
-  const unsigned long long tot = warp_sum_u64((unsigned long long)np);
-  const unsigned long long mx = warp_max_u64((unsigned long long)np);
-  if (lane == 0) { atomicAdd(&s_total, tot); atomicMax(&s_max, mx); }
+  tot = warp_sum_u64(tot);
+  mxnp = warp_max_u64(mxnp);
+  span_max = __reduce_max_sync(0xffffffffu, span_max);
+  if (lane == 0) {
+    if (tot) atomicAdd(&s_total, tot);
+    if (mxnp) atomicMax(&s_max, mxnp);
+    if (span_max > 0) atomicMax(&acc->range_rmax, span_max);
+  }
   __syncthreads();
   if (threadIdx.x < kMaxGroups && s_cnt[threadIdx.x]) atomicAdd(&acc->sym_rows[threadIdx.x], (unsigned long long)s_cnt[threadIdx.x]);
   if (threadIdx.x == 0) {
-    atomicAdd(&acc->total_nprod, s_total);
-    atomicMax(&acc->max_nprod, s_max);
+    if (s_total) atomicAdd(&acc->total_nprod, s_total);
+    if (s_max) atomicMax(&acc->max_nprod, s_max);
   }
 }
 
@@ -393,13 +428,16 @@ cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const i
                                int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
                                int* nlaunch) {
   if (m == 0) return cudaSuccess;
+  // grid-stride kernels: enough CTAs for any lanes-per-row choice (rows / 8 per CTA-pass at G = 32)
+  auto grid_of = [](long long rows) {
+    const long long want = (rows + (kSetupThreads / 32) - 1) / (kSetupThreads / 32);
+    return (unsigned)(want < 148LL * 16 ? (want > 0 ? want : 1) : 148LL * 16);
+  };
   if (bmm && k > 0) {
-    k_brow_minmax<<<(unsigned)((k + kSetupThreads - 1) / kSetupThreads), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm,
-                                                                                               &acc->b_unsorted);
+    k_brow_minmax<<<grid_of(k), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm, &acc->b_unsorted);
     if (nlaunch) ++*nlaunch;
   }
-  const unsigned grid = (unsigned)((m + kSetupThreads - 1) / kSetupThreads);
-  k_nprod_group<<<grid, kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b);
+  k_nprod_group<<<grid_of(m), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b);
   if (nlaunch) ++*nlaunch;
   return cudaGetLastError();
 }

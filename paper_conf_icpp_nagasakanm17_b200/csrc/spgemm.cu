@@ -94,7 +94,7 @@ struct spgemm_ctx {
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
   Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi, num_slab, num_slab_c,
-      rbits;
+      rbits, bbits;
   bool range_num = false;  // numeric range rows on for the last symbolic call (bitmap allocated, B sorted)
   GraphCache gsym, gnum;  // captured segments (see run_graph)
   int use_graphs = 1;
@@ -174,7 +174,7 @@ void release_state(spgemm_handle_t h) {
 
 void free_all(spgemm_handle_t h) {
   Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow,
-                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits};
+                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits, &h->bbits};
   for (Buf* b : all) buf_free(h, *b);
   release_state(h);
 }
@@ -498,7 +498,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_CLUSTER_FILL_LIMIT:
       if (v < 0) return fail(h, SPGEMM_ERR_INVALID_ARG, "CLUSTER_FILL_LIMIT < 0");
       h->cluster_fill = (int)std::min<int64_t>(v, 1 << 30); break;
-    case SPGEMM_OPT_RANGE_WARP: h->range_warp = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANGE_WARP:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_WARP must be 0, 1 or 2");
+      h->range_warp = (int)v; break;
     case SPGEMM_OPT_RANGE_MIN_NPROD:
       if (v < 1 || v > kRangeMaxNprod) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_MIN_NPROD out of range");
       h->range_min_np = v; break;
@@ -619,7 +621,16 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   // range rows: pattern bitmap (symbolic -> numeric gather), rwcap words per row of the group
   const long long n_range = (long long)h->snap1.sym_rows[kSymRange];
   h->range_num = false;
+  int range_bw = 0;  // > 0: symbolic range rows by B-row bitmap union (words per B-row bitmap)
   if (n_range > 0) {
+    if (h->range_warp == 1 && h->snap1.range_rmax <= 1024) {
+      const int bw = range_wcap(h->snap1.range_rmax);
+      const long long bytes = k * (long long)bw * 4;
+      if (bytes <= h->ws_budget / 2) {
+        ALLOC(h->bbits, (size_t)bytes);
+        range_bw = bw;
+      }
+    }
     sa.rwcap = range_wcap(h->snap1.range_rmax);
     const long long bytes = n_range * sa.rwcap * 4;  // <= 256 B per range row
     if (bytes <= h->ws_budget) {
@@ -634,13 +645,14 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   std::vector<long long> topo = {1, m, k, n, glob_grid, slab_T, h->vw_log2, sa.long_len, sa.flat, sa.fill_limit,
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
-                                 h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num};
+                                 h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
                                        (long long)h->slab_sym.p, (long long)h->overflow.p, (long long)h->overflow2.p,
                                        (long long)h->grp2.p, (long long)h->rlohi.p, (long long)h->nprod.p,
-                                       (long long)h->tiles.p, (long long)h->grp1.p, (long long)h->rbits.p};
+                                       (long long)h->tiles.p, (long long)h->grp1.p, (long long)h->rbits.p,
+                                       (long long)h->bbits.p, (long long)h->bmm.p};
   int seg_launches = 0;
   const bool ge = group_events(h);
   h->gtimed_phases = ge && h->timing;
@@ -691,8 +703,16 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       SymArgs ra = sa;
       ra.rows = perm1 + off1.off[kSymRange];
       ra.nrows = (long long)h->snap1.sym_rows[kSymRange];
-      CK(launch_symbolic_range(s, ra, h->snap1.range_rmax, h->num_sms));
-      ++launches;
+      if (range_bw > 0) {  // B-row bitmaps, then the bitmap-union count
+        CK(launch_brow_bits(s, k, b_rpt, b_col, static_cast<const int2*>(h->bmm.p), static_cast<unsigned*>(h->bbits.p),
+                            range_bw, h->num_sms));
+        CK(launch_symbolic_range_bits(s, ra, static_cast<const unsigned*>(h->bbits.p), range_bw,
+                                      static_cast<const int2*>(h->bmm.p), h->num_sms));
+        launches += 2;
+      } else {
+        CK(launch_symbolic_range(s, ra, h->snap1.range_rmax, h->num_sms));
+        ++launches;
+      }
       if (ge) CK(cudaEventRecord(h->gstop[0][kSymRange], s));
       h->gtimed[0][kSymRange] = ge;
     }

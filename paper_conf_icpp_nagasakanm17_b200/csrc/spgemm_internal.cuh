@@ -741,6 +741,10 @@ cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int3
 cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);
 cudaError_t launch_symbolic_range(cudaStream_t s, const SymArgs& a, int rmax, int num_sms);
 cudaError_t launch_numeric_range(cudaStream_t s, bool fp64, const NumArgs& a, int rmax, int num_sms);
+cudaError_t launch_brow_bits(cudaStream_t s, long long k, const int64_t* b_rpt, const int32_t* b_col,
+                             const int2* bmm, unsigned* bbits, int bw, int num_sms);
+cudaError_t launch_symbolic_range_bits(cudaStream_t s, const SymArgs& a, const unsigned* bbits, int bw,
+                                       const int2* bmm, int num_sms);
 int range_warps(long long per_warp);
 int range_rcap(long long rmax);
 int range_wcap(long long rmax);

@@ -339,10 +339,11 @@ RANGE_CASES = ["cant", "mixed:protein", "mixed:accelerator", "mixed:circuit"]
 
 @pytest.mark.parametrize("name", RANGE_CASES)
 @pytest.mark.parametrize("dtype", [np.float32, np.float64])
-def test_range_rows(spg, name, dtype):
+@pytest.mark.parametrize("mode", [1, 2])  # 1: bitmap-union count, 2: per-product flags
+def test_range_rows(spg, name, dtype, mode):
     """Every row that qualifies (min n_prod lowered to 1) through the warp-per-row kernels."""
     A = synth.config(name)
-    got = check(spg, A, A, dtype, opts={"range_min_nprod": 1}, what=f"{name} range rows")
+    got = check(spg, A, A, dtype, opts={"range_min_nprod": 1, "range_warp": mode}, what=f"{name} range rows")
     st = got[3]
     assert st["sym_rows"][spg.SYM_RANGE_GROUP] > 0
     assert st["num_rows"][spg.NUM_RANGE_GROUP] == st["sym_rows"][spg.SYM_RANGE_GROUP]
@@ -381,23 +382,26 @@ def test_range_rows_unsorted_b(spg):
     assert got[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0 and got[3]["num_rows"][spg.NUM_RANGE_GROUP] == 0
 
 
-def test_range_rows_ragged(spg):
-    """Spans that are not multiples of 16/32, rows with a single A entry, empty rows, R = 1."""
+@pytest.mark.parametrize("wmax", [40, 700])
+def test_range_rows_ragged(spg, wmax):
+    """Spans that are not multiples of 16/32, rows with a single A entry, empty rows, R = 1;
+    wmax 700: spans beyond 1024 (flag-store count) and beyond 2048 (not range rows)."""
     rng = np.random.default_rng(11)
     m = 3000
     rows, cols = [], []
     for i in range(m):
         if i % 97 == 0:
             continue  # empty row
-        w = int(rng.integers(0, 40))
+        w = int(rng.integers(0, wmax))
         L = int(rng.integers(1, 2 * w + 2))
         c = np.unique(np.clip(i + rng.integers(-w, w + 1, L), 0, m - 1))
         rows += [i] * len(c)
         cols += c.tolist()
     A = from_coo(m, m, np.array(rows), np.array(cols), name="ragged").with_values("uniform", 12)
     for dtype in (np.float32, np.float64):
-        got = check(spg, A, A, dtype, opts={"range_min_nprod": 1}, what="ragged range")
-        assert got[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0
+        for mode in (1, 2):
+            got = check(spg, A, A, dtype, opts={"range_min_nprod": 1, "range_warp": mode}, what="ragged range")
+            assert got[3]["sym_rows"][spg.SYM_RANGE_GROUP] > 0
 
 
 # ------------------------------------------------------------------ intermediate steps
