@@ -153,7 +153,10 @@ typedef enum {
                                        per product.  2: range rows, flag stores always (ablation).
                                        0: Table-I groups only.  Needs RANGE_HASH; off while a
                                        MIN_GROUP is forced */
-    SPGEMM_OPT_RANGE_MIN_NPROD = 15 /* n_prod lower bound of range rows (default 256) */
+    SPGEMM_OPT_RANGE_MIN_NPROD = 15,/* n_prod lower bound of range rows (default 256) */
+    SPGEMM_OPT_BITMAP_RANK = 16     /* 1 (default): CTA-per-row numeric groups order each row by a
+                                       two-level bitmap rank over its column span;
+                                       0: bucket sort (ablation) */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

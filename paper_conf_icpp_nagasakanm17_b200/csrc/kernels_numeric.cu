@@ -46,9 +46,9 @@ struct Vec16<double> { using T = double2; static __device__ __forceinline__ doub
 
 // The product loop of one numeric row: CTA-per-row groups in flat mode use the block-level
 // flattened loop; otherwise the per-sub-group loop plus the CTA pass over deferred long B rows.
-template <int TPR, typename VT, typename F>
+template <int TPR, typename VT, typename BF, typename F>
 __device__ __forceinline__ void num_products(const NumArgs& a, bool active, int row, int t, int long_len, int* s_list,
-                                             int* s_lcnt, BlockFlat<VT>* bf, long long* ws, F&& f) {
+                                             int* s_lcnt, BF* bf, long long* ws, F&& f) {
   const VT* av = static_cast<const VT*>(a.a_val);
   const VT* bv = static_cast<const VT*>(a.b_val);
   if constexpr (TPR > 32) {
@@ -68,13 +68,107 @@ __device__ __forceinline__ void num_products(const NumArgs& a, bool active, int 
   }
 }
 
+// Scratch of the two-level bitmap rank (CTA-per-row groups).
+struct Rank2 {
+  unsigned* fine;    // [upper] bits of the non-empty 32-column blocks, compacted
+  uint16_t* pre2;    // [upper] exclusive prefix popcount of fine (rank of the block's first key)
+  unsigned* l1;      // [l1_words] level-1 bitmap: bit = 32-column block is non-empty
+  unsigned* p1;      // [l1_words] exclusive prefix popcount of l1 (compact index of a block)
+};
+
+// Shared atomicOr of one key's bit (ATOMS.OR; a software peer reduction with a partial-warp
+// __reduce_or_sync mask measured 3x slower than letting the atomic unit serialise same-word lanes).
+__device__ __forceinline__ void or_aggregated(bool valid, unsigned* base, int idx, unsigned bits) {
+  if (valid) atomicOr(base + idx, bits);
+}
+
+// (c) for CTA-per-row groups: rank of every key = number of smaller keys of the row, from a
+// two-level bitmap over [lo, hi]: level 1 marks the non-empty 32-column blocks
+// (R/1024 words), its prefix popcount gives each non-empty block a compact index b, level 2
+// holds the 32-bit pattern of block b, and rank(key) = pre2[b] + popc(fine[b] & below(key)).
+// O(n + R/1024) work, no sorting, no crowding (a dense cluster only fills level-2 words).  Keys
+// are distinct, so the result is the unique ascending order.  T/4 is a multiple
+// of TPR in every CTA group, so the slot loops are warp-uniform (match_any needs full warps).
+template <typename VT, int TPR>
+__device__ __forceinline__ long long rank_write_2level(const int* Kp, const VT* Vp, unsigned T, int lo, int hi,
+                                                       const Rank2& r2, long long* ws, bool active, int32_t* cc,
+                                                       VT* cv, long long cn) {
+  const int t = threadIdx.x;
+  const int4* k4 = reinterpret_cast<const int4*>(Kp);
+  const int W1 = hi >= lo ? (int)(((unsigned)(hi - lo)) >> 10) + 1 : 0;
+  for (int w = t; w < W1; w += TPR) r2.l1[w] = 0u;
+  __syncthreads();
+  for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+    const int4 kv = k4[s4];
+    const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const unsigned d = (unsigned)(ks[u] - lo);
+      or_aggregated(ks[u] >= 0, r2.l1, (int)(d >> 10), 1u << ((d >> 5) & 31));
+    }
+  }
+  __syncthreads();
+  long long nb = 0;
+  {
+    const int per = (W1 + TPR - 1) / TPR;
+    const int w0 = t * per, w1 = min(W1, w0 + per);
+    long long loc = 0;
+    for (int w = w0; w < w1; ++w) loc += __popc(r2.l1[w]);
+    long long run = Grp<TPR>::excl_scan(loc, &nb, ws);
+    for (int w = w0; w < w1; ++w) { r2.p1[w] = (unsigned)run; run += __popc(r2.l1[w]); }
+  }
+  for (int b = t; b < (int)nb; b += TPR) r2.fine[b] = 0u;
+  __syncthreads();
+  auto block_of = [&](unsigned d) {
+    const unsigned w = d >> 10, bit = (d >> 5) & 31;
+    return (int)(r2.p1[w] + __popc(r2.l1[w] & ((1u << bit) - 1u)));
+  };
+  for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+    const int4 kv = k4[s4];
+    const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const unsigned d = (unsigned)(ks[u] - lo);
+      const bool valid = ks[u] >= 0;
+      or_aggregated(valid, r2.fine, valid ? block_of(d) : 0, 1u << (d & 31));
+    }
+  }
+  __syncthreads();
+  long long n_total = 0;
+  {
+    const int per = (int)((nb + TPR - 1) / TPR);
+    const int b0 = t * per, b1 = min((int)nb, b0 + per);
+    long long loc = 0;
+    for (int b = b0; b < b1; ++b) loc += __popc(r2.fine[b]);
+    long long run = Grp<TPR>::excl_scan(loc, &n_total, ws);
+    for (int b = b0; b < b1; ++b) { r2.pre2[b] = (uint16_t)run; run += __popc(r2.fine[b]); }
+  }
+  __syncthreads();
+  if (active) {
+    for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
+      const int4 kv = k4[s4];
+      const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        if (ks[u] < 0) continue;
+        const unsigned d = (unsigned)(ks[u] - lo);
+        const int b = block_of(d);
+        const long long r = (long long)r2.pre2[b] + __popc(r2.fine[b] & ((1u << (d & 31)) - 1u));
+        if (r < cn) { cc[r] = ks[u]; cv[r] = Vp[4 * s4 + u]; }
+      }
+    }
+  }
+  return n_total;
+}
+
 // One row: (0) init, (a) accumulate, (b) gather into buckets, (c) rank + write.
 // Kp/Vp: the key/value tables (shared or global); Keys/Vals: their probe/add accessors.
-template <typename VT, int TPR, bool GLOBAL, typename Keys, typename Vals, typename SIdx>
+template <typename VT, int TPR, bool GLOBAL, bool RANK2 = false, typename Keys, typename Vals, typename SIdx,
+          typename BF>
 __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, const Keys& K, const Vals& V,
                                         int* Kp, VT* Vp, int* Bc, SIdx* S, unsigned mask, int NB, int* lohi,
                                         long long* ws, int* s_list, int* s_lcnt, unsigned* wscr,
-                                        BlockFlat<VT>* bf) {
+                                        BF* bf, const Rank2& r2 = Rank2{}) {
   const int t = Grp<TPR>::lane();
   const unsigned T = mask + 1;
   if (TPR > 32 && t == 0) *s_lcnt = 0;  // pass-1 "deferred a long row" flag (read after a barrier)
@@ -166,7 +260,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
           st_s8(kb + d, 1);
           V.add(d, prod);
         };
-        num_products<TPR>(a, true, row, t, long_len, s_list, s_lcnt, bf, ws, f);
+        num_products<TPR, VT>(a, true, row, t, long_len, s_list, s_lcnt, bf, ws, f);
         Grp<TPR>::sync();
         // in-order compaction: thread owns a contiguous run of flag words
         const int pw = (words + TPR - 1) / TPR;
@@ -208,7 +302,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
       V.add(s, prod);
     };
     const int long_len = TPR > 32 ? a.long_len : 0;
-    num_products<TPR>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f);
+    num_products<TPR, VT>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f);
   }
   Grp<TPR>::sync();
 
@@ -266,6 +360,9 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
         if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
       }
     }
+  } else if constexpr (RANK2) {
+    n_total = rank_write_2level<VT, TPR>(Kp, Vp, T, lo, hi, r2, ws, active, cc, cv, cn);
+    if (t == 0 && active && cn != n_total) atomicOr(a.err_flags, 2);
   } else {
     int shift = 0, nb = 0;
     if (hi >= lo) {
@@ -446,7 +543,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
   Grp<TPR>::sync();
 }
 
-template <typename VT, int T, int TPR, int BS, long long UPPER>
+template <typename VT, int T, int TPR, int BS, long long UPPER, bool RANK2>
 __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ long long ws[33];
@@ -456,8 +553,8 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   // per-warp bucket bitmap+prefix of the (c4) sort, aliased with the block-flat product scratch
   // (used in different phases of a row; separated by barriers)
   constexpr int kWscrBytes = TPR > 32 ? (TPR / 32) * 8 * kWarpBitmapWords<TPR> : 4;
-  constexpr int kAuxBytes = TPR > 32 ? (kWscrBytes > (int)sizeof(BlockFlat<VT>) ? kWscrBytes : (int)sizeof(BlockFlat<VT>))
-                                     : 4;
+  using BF = BlockFlat<VT, RANK2 ? flat_chunk_of<TPR>() : kFlatChunk>;
+  constexpr int kAuxBytes = TPR > 32 ? (kWscrBytes > (int)sizeof(BF) ? kWscrBytes : (int)sizeof(BF)) : 4;
   __shared__ __align__(16) unsigned char s_aux[kAuxBytes];
   unsigned* s_wscr = reinterpret_cast<unsigned*>(s_aux);
   constexpr int NB = num_nbuckets(T);
@@ -471,8 +568,20 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   const long long ridx = (long long)blockIdx.x * RPB + g;
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : 0;
-  num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
-                          s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr, reinterpret_cast<BlockFlat<VT>*>(s_aux));
+  if constexpr (RANK2) {
+    static_assert(TPR == BS, "two-level rank: one row per CTA");
+    Rank2 r2;
+    r2.fine = reinterpret_cast<unsigned*>(Kp + T);
+    r2.pre2 = reinterpret_cast<uint16_t*>(r2.fine + UPPER);
+    r2.l1 = reinterpret_cast<unsigned*>(smem_raw + align16(T * (int)sizeof(VT) + T * 4 + (int)UPPER * 6));
+    r2.p1 = r2.l1 + a.l1_words;
+    num_row<VT, TPR, false, true>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp,
+                                  reinterpret_cast<int*>(r2.fine), (uint16_t*)nullptr, T - 1, NB, s_lohi, ws, s_list,
+                                  &s_lcnt, s_wscr, reinterpret_cast<BF*>(s_aux), r2);
+  } else {
+    num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
+                            s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr, reinterpret_cast<BF*>(s_aux));
+  }
 }
 
 template <typename VT>
@@ -497,27 +606,57 @@ __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
   }
 }
 
-template <typename VT, int T, int TPR, int BS, long long UPPER>
-cudaError_t launch_num(cudaStream_t s, const NumArgs& a) {
-  constexpr int RPB = BS / TPR;
-  constexpr int smem = RPB * num_row_bytes<VT>(T, UPPER);
-  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 +
-                    (TPR > 32 ? (TPR / 32 * 8 * kWarpBitmapWords<TPR> > (int)sizeof(BlockFlat<VT>)
-                                     ? TPR / 32 * 8 * kWarpBitmapWords<TPR> : (int)sizeof(BlockFlat<VT>)) : 4) <= kSmemLimit,
-                "numeric table too large");
-  static bool configured = false;
-  if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(k_num_smem<VT, T, TPR, BS, UPPER>,
+template <typename VT, int T, int TPR, int BS, long long UPPER, bool RANK2>
+cudaError_t launch_num_k(cudaStream_t s, const NumArgs& a, int smem) {
+  static int configured = 0;
+  if (smem > configured) {
+    cudaError_t e = cudaFuncSetAttribute(k_num_smem<VT, T, TPR, BS, UPPER, RANK2>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    configured = true;
+    configured = smem;
   }
   NumArgs b = a;
   const int max_vw = TPR < 32 ? TPR : 32;
   while ((1 << b.vw_log2) > max_vw) --b.vw_log2;
+  constexpr int RPB = BS / TPR;
   const long long grid = (a.nrows + RPB - 1) / RPB;
-  k_num_smem<VT, T, TPR, BS, UPPER><<<(unsigned)grid, BS, smem, s>>>(b);
+  k_num_smem<VT, T, TPR, BS, UPPER, RANK2><<<(unsigned)grid, BS, smem, s>>>(b);
   return cudaGetLastError();
+}
+
+// static shared memory of k_num_smem besides the dynamic tables
+template <typename VT, int TPR>
+constexpr int num_static_bytes() {
+  return 33 * 8 + 8 * 32 + 4 * kLongChunk + 16 +
+         (TPR > 32 ? (TPR / 32 * 8 * kWarpBitmapWords<TPR> > (int)sizeof(BlockFlat<VT, flat_chunk_of<TPR>()>)
+                          ? TPR / 32 * 8 * kWarpBitmapWords<TPR>
+                          : (int)sizeof(BlockFlat<VT, flat_chunk_of<TPR>()>))
+                   : 4);
+}
+
+template <typename VT, int T, int TPR, int BS, long long UPPER>
+cudaError_t launch_num_old(cudaStream_t s, const NumArgs& a);
+
+template <typename VT, int T, int TPR, int BS, long long UPPER>
+cudaError_t launch_num(cudaStream_t s, const NumArgs& a) {
+  if constexpr (TPR > 32) {  // CTA per row: two-level bitmap rank when its scratch fits
+    const long long smem2 = num_cta_bytes<VT>(T, UPPER, a.l1_words);
+    if (a.l1_words > 0 && smem2 + num_static_bytes<VT, TPR>() <= kSmemLimit)
+      return launch_num_k<VT, T, TPR, BS, UPPER, true>(s, a, (int)smem2);
+  }
+  return launch_num_old<VT, T, TPR, BS, UPPER>(s, a);
+}
+
+template <typename VT, int T, int TPR, int BS, long long UPPER>
+cudaError_t launch_num_old(cudaStream_t s, const NumArgs& a) {
+  constexpr int RPB = BS / TPR;
+  constexpr int smem = RPB * num_row_bytes<VT>(T, UPPER);
+  static_assert(smem + 33 * 8 + 8 * RPB + 4 * kLongChunk + 16 +
+                    (TPR > 32 ? (TPR / 32 * 8 * kWarpBitmapWords<TPR> > (int)sizeof(BlockFlat<VT>)
+                                     ? TPR / 32 * 8 * kWarpBitmapWords<TPR>
+                                     : (int)sizeof(BlockFlat<VT>)) : 4) <= kSmemLimit,
+                "numeric table too large");
+  return launch_num_k<VT, T, TPR, BS, UPPER, false>(s, a, smem);
 }
 
 template <typename VT>

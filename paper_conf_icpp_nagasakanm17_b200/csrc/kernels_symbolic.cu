@@ -27,9 +27,9 @@ struct NoStop {
 
 // The product loop of one symbolic row: CTA-per-row groups in flat mode use the block-level
 // flattened loop; otherwise the per-sub-group loop plus the CTA pass over deferred long B rows.
-template <bool STOP, int TPR, typename F, typename S>
+template <bool STOP, int TPR, typename BF, typename F, typename S>
 __device__ __forceinline__ void sym_products(const SymArgs& a, bool active, int row, int t, int long_len,
-                                             int* s_list, int& s_lcnt, BlockFlat<int>* bf, long long* ws, F&& f,
+                                             int* s_list, int& s_lcnt, BF* bf, long long* ws, F&& f,
                                              S&& stop) {
   if constexpr (TPR > 32) {
     if (a.flat) {
@@ -49,9 +49,9 @@ __device__ __forceinline__ void sym_products(const SymArgs& a, bool active, int 
 }
 
 // One row (all TPR threads of its row group call it; the table is the group's slice).
-template <int T, int TPR, bool OPT>
+template <int T, int TPR, bool OPT, typename BF>
 __device__ __forceinline__ void sym_row(const SymArgs& a, bool active, int row, int t, int* table, long long* ws,
-                                        int& s_cnt, int& s_abort, int& s_lcnt, int* s_list, BlockFlat<int>* bf) {
+                                        int& s_cnt, int& s_abort, int& s_lcnt, int* s_list, BF* bf) {
   // Range-offset hash: when the row's column span R fits 4*T bytes the table
   // is a byte-flag array indexed by key - lo_i (collision-free; idempotent plain stores, no
   // atomics, conflict-free for consecutive keys); the count is the number of set flags.
@@ -132,7 +132,8 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_cnt, s_abort, s_lcnt;
   __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
-  __shared__ std::conditional_t<(TPR > 32), BlockFlat<int>, int> s_bf_store;  // only CTA groups need it
+  using BF = BlockFlat<int, flat_chunk_of<TPR>()>;
+  __shared__ std::conditional_t<(TPR > 32), BF, int> s_bf_store;  // only CTA groups need it
   constexpr int RPB = BS / TPR;
   static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");
   const int g = threadIdx.x / TPR, t = threadIdx.x % TPR;
@@ -141,7 +142,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   const bool active = ridx < a.nrows;
   const int row = active ? a.rows[ridx] : -1;
   sym_row<T, TPR, OPT>(a, active, row, t, table, ws, s_cnt, s_abort, s_lcnt, s_list,
-                       reinterpret_cast<BlockFlat<int>*>(&s_bf_store));
+                       reinterpret_cast<BF*>(&s_bf_store));
 }
 
 // Global-memory table per CTA (slab of slab_T ints), one row at a time; table size

@@ -84,6 +84,7 @@ struct spgemm_ctx {
   int timing = 1;
   int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
   long long range_min_np = kRangeMinNprodDefault;
+  int bitmap_rank = 1;   // CTA-per-row numeric groups: two-level bitmap rank (else bucket sort)
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
   int state = 0;
@@ -504,6 +505,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_RANGE_MIN_NPROD:
       if (v < 1 || v > kRangeMaxNprod) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_MIN_NPROD out of range");
       h->range_min_np = v; break;
+    case SPGEMM_OPT_BITMAP_RANK: h->bitmap_rank = v ? 1 : 0; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -823,6 +825,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.rlohi = static_cast<const int2*>(h->rlohi.p);
     na.priv_ok = h->snap1.b_unsorted ? 0 : 1;
     na.err_flags = &dacc->err_flags;
+    na.l1_words = h->bitmap_rank ? (int)((h->n + 1023) / 1024 + 1) : 0;
     // cluster groups (clusters of 2/4/8 CTAs): bitmap + prefix scratch per resident cluster
     const long long cwords = h->n / 32 + 2;
     const long long cstride = (2 * cwords * 4 + 255) & ~255LL;
@@ -854,7 +857,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // numeric re-runs with new values of the same structure, or repeated multiplies)
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
-                                   h->snap1.range_rmax};
+                                   h->snap1.range_rmax, (long long)na.l1_words};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,

@@ -92,6 +92,12 @@ template <typename VT>
 __host__ __device__ constexpr int num_row_bytes(int T, long long upper) {
   return align16(T * (int)sizeof(VT) + T * 4 + (num_nbuckets(T) + 1) * 4 + (int)upper * 2 + 8);
 }
+// CTA-per-row numeric groups with the two-level bitmap rank (kernels_numeric.cu):
+// vals[T] | keys[T] | fine[upper] u32 | pre2[upper] u16 | lvl1[l1] u32 | pre1[l1] u32
+template <typename VT>
+__host__ __device__ constexpr long long num_cta_bytes(int T, long long upper, long long l1) {
+  return align16(T * (int)sizeof(VT) + T * 4 + (int)upper * 6) + l1 * 8 + 16;
+}
 
 // ----------------------------------------------------------------------------- device state
 struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned host at the syncs
@@ -350,23 +356,28 @@ __device__ __forceinline__ void for_each_product_flat(const int64_t* __restrict_
 constexpr int kFlatChunk = 256;
 template <int TPR>
 struct Grp;  // row-group collectives (defined below)
-template <typename VT>
+// N entries per chunk: kFlatChunk by default; the CTA-per-row group kernels use one chunk of TPR
+// entries (up to 1024) so that a row of <= TPR A non-zeros costs a single metadata round trip.
+template <typename VT, int N = kFlatChunk>
 struct BlockFlat {
-  long long b0[kFlatChunk];
-  int incl[kFlatChunk];
-  VT av[kFlatChunk];
+  static constexpr int kN = N;
+  long long b0[N];
+  int incl[N];
+  VT av[N];
 };
-template <bool NUM, bool CHECK_STOP, typename VT, int TPR, typename F, typename S>
+template <int TPR>
+constexpr int flat_chunk_of() { return TPR < 1024 ? TPR : 1024; }
+template <bool NUM, bool CHECK_STOP, typename VT, int TPR, typename BF, typename F, typename S>
 __device__ __forceinline__ void for_each_product_block(const int64_t* __restrict__ a_rpt,
                                                        const int32_t* __restrict__ a_col,
                                                        const VT* __restrict__ a_val,
                                                        const int64_t* __restrict__ b_rpt,
                                                        const int32_t* __restrict__ b_col,
                                                        const VT* __restrict__ b_val, bool active, int row, int t,
-                                                       BlockFlat<VT>* sh, long long* ws, F&& f, S&& stop,
+                                                       BF* sh, long long* ws, F&& f, S&& stop,
                                                        int part = 0, int nparts = 1) {
   static_assert(TPR > 32, "CTA-level loop");
-  constexpr int CH = TPR < kFlatChunk ? TPR : kFlatChunk;
+  constexpr int CH = TPR < BF::kN ? TPR : BF::kN;
   constexpr int tpr = TPR;
   const long long a0 = active ? __ldg(a_rpt + row) : 0;
   const int na = active ? (int)(__ldg(a_rpt + row + 1) - a0) : 0;  // CTA-uniform
@@ -435,12 +446,12 @@ __device__ __forceinline__ void products(bool flat, const int64_t* __restrict__ 
 // one B row) walks the listed rows one at a time instead.  A stopped (CHECK_STOP) thread keeps
 // hitting barriers.
 constexpr int kLongChunk = 256;
-template <bool NUM, bool CHECK_STOP, typename VT, bool WSYNC = false, typename F, typename S>
+template <bool NUM, bool CHECK_STOP, typename VT, bool WSYNC = false, typename BF, typename F, typename S>
 __device__ __forceinline__ void for_long_products(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
                                                   const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
                                                   const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
                                                   bool active, int row, int t, int tpr, int long_len, int* s_list,
-                                                  int* s_cnt, BlockFlat<VT>* bf, F&& f, S&& stop, int part = 0,
+                                                  int* s_cnt, BF* bf, F&& f, S&& stop, int part = 0,
                                                   int nparts = 1) {
   const long long a0 = active ? __ldg(a_rpt + row) : 0;
   const int32_t* __restrict__ ac = a_col + a0;
@@ -712,6 +723,7 @@ struct NumArgs {
   // global fallback
   void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;
   const unsigned* rbits; long long rwcap;  // range rows: symbolic pattern bitmap (same row order)
+  int l1_words;            // CTA-per-row groups: level-1 words of the two-level rank (>= n/1024 + 1)
 };
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,

@@ -136,11 +136,25 @@ def test_forced_symbolic_group(spg, group, range_hash):
 
 @pytest.mark.parametrize("range_hash", [0, 1])
 @pytest.mark.parametrize("group", list(range(0, 14)))
-def test_forced_numeric_group(spg, group, range_hash):
+@pytest.mark.parametrize("bitmap_rank", [1, 0])  # CTA groups: two-level bitmap rank / bucket sort
+def test_forced_numeric_group(spg, group, range_hash, bitmap_rank):
+    if bitmap_rank == 0 and not 4 <= group <= 9:
+        pytest.skip("bucket sort ablation only differs in the CTA-per-row groups")
     for A in (_mixed_small(), _banded_small()):
         ref = oracle.spgemm(A, A, np.float32)
-        got = run_gpu(spg, A, A, np.float32, {"num_min_group": group, "range_hash": range_hash})
+        got = run_gpu(spg, A, A, np.float32, {"num_min_group": group, "range_hash": range_hash,
+                                              "bitmap_rank": bitmap_rank})
         assert_parity(got, ref, np.float32, what=f"{A.name} num group>={group} range_hash={range_hash}")
+
+
+@pytest.mark.parametrize("group", [4, 6, 8, 9])
+def test_bitmap_rank_dense_clusters_f64(spg, group):
+    """Two-level bitmap rank on rows whose keys form dense clusters plus far outliers (webbase
+    shape), fp64 (group 9 fp64 exceeds shared memory with the rank scratch: bucket sort)."""
+    A = synth.config("webbase", "int")
+    A = oracle.row_slice(A, 0, 60000)
+    B = synth.config("webbase", "int")
+    got = check(spg, A, B, np.float64, exact=True, opts={"num_min_group": group}, what=f"dense clusters g{group}")
 
 
 @pytest.mark.parametrize("config", ["cant", "webbase", "mixed:protein", "mixed:economics"])
