@@ -140,8 +140,20 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
   const CKeys K{s_kp, 31 - __clz(Ts), Ts - 1};
   const CVals<VT> V{s_vp, 31 - __clz(Ts), Ts - 1};
   const unsigned mask = CS * Ts - 1;
-  for (long long i = cid; i < a.nrows; i += nclusters) {
+  // rows are handed out dynamically (one global counter per launch; rank 0 fetches, the cluster
+  // reads it through DSMEM): row costs vary by 10x within a group (measured 3x span/mean imbalance
+  // with the static cid-strided assignment)
+  __shared__ long long s_next;
+  const long long* next0 = cluster.map_shared_rank(&s_next, 0);
+  (void)nclusters; (void)cid;
+  while (true) {
+    if (rank == 0 && t == 0) s_next = a.row_counter ? (long long)atomicAdd(a.row_counter, 1) : 0;
+    cluster.sync();
+    const long long i = *(volatile const long long*)next0;
+    cluster.sync();  // every CTA has read it: rank 0 may overwrite it or exit
+    if (i >= a.nrows) break;  // cluster-uniform
     const int row = a.rows[i];
+    if (a.prof && rank == 0 && t == 0) a.prof[4 * i + 1] = gtimer();
     int4* k4 = reinterpret_cast<int4*>(Kloc);
     for (int s = t; s < Ts / 4; s += 1024) k4[s] = make_int4(-1, -1, -1, -1);
     for (int s = t; s < Ts; s += 1024) Vloc[s] = VT(0);
@@ -165,6 +177,7 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
                                          &s_lcnt, &s_bf, f, NoStop{}, rank, CS);
     }
     cluster.sync();
+    if (a.prof && rank == 0 && t == 0) a.prof[4 * i + 2] = gtimer();
     // (b) column span of the row: min/max over every slice, reduced into CTA 0
     {
       int mn = INT_MAX, mx = -1;
@@ -241,6 +254,12 @@ __global__ void __launch_bounds__(1024) k_num_cluster(NumArgs a) {
       if (r < cn) { cc[r] = k; cv[r] = Vloc[s]; }
     }
     cluster.sync();
+    if (a.prof && rank == 0 && t == 0) {
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      a.prof[4 * i + 3] = gtimer();
+      a.prof[4 * i + 0] = ((unsigned long long)smid << 32) | (unsigned)row;
+    }
   }
 }
 

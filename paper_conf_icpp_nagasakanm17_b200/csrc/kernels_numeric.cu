@@ -82,30 +82,55 @@ __device__ __forceinline__ void or_aggregated(bool valid, unsigned* base, int id
   if (valid) atomicOr(base + idx, bits);
 }
 
-// (c) for CTA-per-row groups: rank of every key = number of smaller keys of the row, from a
-// two-level bitmap over [lo, hi]: level 1 marks the non-empty 32-column blocks
-// (R/1024 words), its prefix popcount gives each non-empty block a compact index b, level 2
-// holds the 32-bit pattern of block b, and rank(key) = pre2[b] + popc(fine[b] & below(key)).
-// O(n + R/1024) work, no sorting, no crowding (a dense cluster only fills level-2 words).  Keys
-// are distinct, so the result is the unique ascending order.  T/4 is a multiple
-// of TPR in every CTA group, so the slot loops are warp-uniform (match_any needs full warps).
-template <typename VT, int TPR>
-__device__ __forceinline__ long long rank_write_2level(const int* Kp, const VT* Vp, unsigned T, int lo, int hi,
-                                                       const Rank2& r2, long long* ws, bool active, int32_t* cc,
-                                                       VT* cv, long long cn) {
+// (b)+(c) for CTA-per-row groups.  (b) gather: every thread takes its T/TPR contiguous slots into
+// registers, the occupied ones are compacted to the front of the table (block scan; the table is
+// no longer probed) and the row's column range [lo, hi] is reduced on the way.  (c) rank of every
+// key = number of smaller keys of the row, from a two-level bitmap over [lo, hi]:
+// level 1 marks the non-empty 32-column blocks (R/1024 words), its prefix popcount gives each
+// non-empty block a compact index b, level 2 holds the 32-bit pattern of block b, and
+// rank(key) = pre2[b] + popc(fine[b] & below(key)).  O(n + R/1024) work on the n compacted keys
+// (KPT = upper/TPR per thread, kept in registers), no sorting, no crowding (a dense cluster only
+// fills level-2 words).  Keys are distinct: the result is the unique ascending order.
+template <typename VT, int TPR, int T, int KPT>
+__device__ __forceinline__ long long gather_rank_2level(int* Kp, VT* Vp, const Rank2& r2, long long* ws, int* lohi,
+                                                        bool active, int32_t* cc, VT* cv, long long cn) {
+  constexpr int SPT = T / TPR;  // slots per thread, a multiple of 4
+  static_assert(SPT % 4 == 0, "slots per thread");
   const int t = threadIdx.x;
-  const int4* k4 = reinterpret_cast<const int4*>(Kp);
+  int ks[SPT];
+  VT vs[SPT];
+  int cnt = 0, mn = INT_MAX, mx = -1;
+  {
+    const int4* k4 = reinterpret_cast<const int4*>(Kp + t * SPT);
+#pragma unroll
+    for (int i = 0; i < SPT / 4; ++i) {
+      const int4 kv = k4[i];
+      ks[4 * i] = kv.x; ks[4 * i + 1] = kv.y; ks[4 * i + 2] = kv.z; ks[4 * i + 3] = kv.w;
+    }
+#pragma unroll
+    for (int i = 0; i < SPT; ++i) {
+      vs[i] = Vp[t * SPT + i];
+      if (ks[i] >= 0) { ++cnt; mn = min(mn, ks[i]); mx = max(mx, ks[i]); }
+    }
+  }
+  long long n;
+  int off = (int)Grp<TPR>::excl_scan(cnt, &n, ws);  // its barriers order the reads before the writes
+  Grp<TPR>::minmax(mn, mx, lohi);
+#pragma unroll
+  for (int i = 0; i < SPT; ++i)
+    if (ks[i] >= 0) { Kp[off] = ks[i]; Vp[off] = vs[i]; ++off; }
+  const int lo = lohi[0], hi = lohi[1];
   const int W1 = hi >= lo ? (int)(((unsigned)(hi - lo)) >> 10) + 1 : 0;
   for (int w = t; w < W1; w += TPR) r2.l1[w] = 0u;
   __syncthreads();
-  for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
-    const int4 kv = k4[s4];
-    const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
+  int kk[KPT];
+  unsigned dd[KPT];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const unsigned d = (unsigned)(ks[u] - lo);
-      or_aggregated(ks[u] >= 0, r2.l1, (int)(d >> 10), 1u << ((d >> 5) & 31));
-    }
+  for (int m = 0; m < KPT; ++m) {
+    const int j = t + m * TPR;
+    kk[m] = j < n ? Kp[j] : -1;
+    dd[m] = (unsigned)(kk[m] - lo);
+    if (kk[m] >= 0) atomicOr(r2.l1 + (dd[m] >> 10), 1u << ((dd[m] >> 5) & 31));
   }
   __syncthreads();
   long long nb = 0;
@@ -119,19 +144,13 @@ __device__ __forceinline__ long long rank_write_2level(const int* Kp, const VT* 
   }
   for (int b = t; b < (int)nb; b += TPR) r2.fine[b] = 0u;
   __syncthreads();
-  auto block_of = [&](unsigned d) {
-    const unsigned w = d >> 10, bit = (d >> 5) & 31;
-    return (int)(r2.p1[w] + __popc(r2.l1[w] & ((1u << bit) - 1u)));
-  };
-  for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
-    const int4 kv = k4[s4];
-    const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
+  int bb[KPT];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const unsigned d = (unsigned)(ks[u] - lo);
-      const bool valid = ks[u] >= 0;
-      or_aggregated(valid, r2.fine, valid ? block_of(d) : 0, 1u << (d & 31));
-    }
+  for (int m = 0; m < KPT; ++m) {
+    if (kk[m] < 0) continue;
+    const unsigned w = dd[m] >> 10, bit = (dd[m] >> 5) & 31;
+    bb[m] = (int)(r2.p1[w] + __popc(r2.l1[w] & ((1u << bit) - 1u)));
+    atomicOr(r2.fine + bb[m], 1u << (dd[m] & 31));
   }
   __syncthreads();
   long long n_total = 0;
@@ -145,17 +164,11 @@ __device__ __forceinline__ long long rank_write_2level(const int* Kp, const VT* 
   }
   __syncthreads();
   if (active) {
-    for (unsigned s4 = t; s4 < T / 4; s4 += TPR) {
-      const int4 kv = k4[s4];
-      const int ks[4] = {kv.x, kv.y, kv.z, kv.w};
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        if (ks[u] < 0) continue;
-        const unsigned d = (unsigned)(ks[u] - lo);
-        const int b = block_of(d);
-        const long long r = (long long)r2.pre2[b] + __popc(r2.fine[b] & ((1u << (d & 31)) - 1u));
-        if (r < cn) { cc[r] = ks[u]; cv[r] = Vp[4 * s4 + u]; }
-      }
+    for (int m = 0; m < KPT; ++m) {
+      if (kk[m] < 0) continue;
+      const long long r = (long long)r2.pre2[bb[m]] + __popc(r2.fine[bb[m]] & ((1u << (dd[m] & 31)) - 1u));
+      if (r < cn) { cc[r] = kk[m]; cv[r] = Vp[t + m * TPR]; }
     }
   }
   return n_total;
@@ -163,8 +176,8 @@ __device__ __forceinline__ long long rank_write_2level(const int* Kp, const VT* 
 
 // One row: (0) init, (a) accumulate, (b) gather into buckets, (c) rank + write.
 // Kp/Vp: the key/value tables (shared or global); Keys/Vals: their probe/add accessors.
-template <typename VT, int TPR, bool GLOBAL, bool RANK2 = false, typename Keys, typename Vals, typename SIdx,
-          typename BF>
+template <typename VT, int TPR, bool GLOBAL, bool RANK2 = false, int TT = 0, int KPT = 0, typename Keys,
+          typename Vals, typename SIdx, typename BF>
 __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, const Keys& K, const Vals& V,
                                         int* Kp, VT* Vp, int* Bc, SIdx* S, unsigned mask, int NB, int* lohi,
                                         long long* ws, int* s_list, int* s_lcnt, unsigned* wscr,
@@ -305,6 +318,22 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
     num_products<TPR, VT>(a, active, row, t, long_len, s_list, s_lcnt, bf, ws, f);
   }
   Grp<TPR>::sync();
+  if constexpr (RANK2) {
+    if (a.prof && threadIdx.x == 0) a.prof[4 * blockIdx.x + 2] = gtimer();
+    const long long c0 = active ? a.c_rpt[row] : 0;
+    const long long cn = active ? a.c_rpt[row + 1] - c0 : 0;
+    const long long n_total = gather_rank_2level<VT, TPR, TT, KPT>(Kp, Vp, r2, ws, lohi, active, a.c_col + c0,
+                                                                   static_cast<VT*>(a.c_val) + c0, cn);
+    if (t == 0 && active && cn != n_total) atomicOr(a.err_flags, 2);
+    Grp<TPR>::sync();
+    if (a.prof && threadIdx.x == 0) {
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      a.prof[4 * blockIdx.x + 3] = gtimer();
+      a.prof[4 * blockIdx.x + 0] = ((unsigned long long)smid << 32) | (unsigned)row;
+    }
+    return;
+  }
 
   // (b) gather: column range [lo, hi] of the row (group min/max over the table)
   const int4* k4 = reinterpret_cast<const int4*>(Kp);
@@ -360,9 +389,6 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
         if (r < cn) { cc[r] = key; cv[r] = Vp[s]; }
       }
     }
-  } else if constexpr (RANK2) {
-    n_total = rank_write_2level<VT, TPR>(Kp, Vp, T, lo, hi, r2, ws, active, cc, cv, cn);
-    if (t == 0 && active && cn != n_total) atomicOr(a.err_flags, 2);
   } else {
     int shift = 0, nb = 0;
     if (hi >= lo) {
@@ -544,7 +570,7 @@ __device__ __forceinline__ void num_row(const NumArgs& a, bool active, int row, 
 }
 
 template <typename VT, int T, int TPR, int BS, long long UPPER, bool RANK2>
-__global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
+__global__ __launch_bounds__(BS, (RANK2 && BS >= 512) ? 2048 / BS : 1) void k_num_smem(NumArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ long long ws[33];
   constexpr int RPB = BS / TPR;
@@ -553,8 +579,11 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   // per-warp bucket bitmap+prefix of the (c4) sort, aliased with the block-flat product scratch
   // (used in different phases of a row; separated by barriers)
   constexpr int kWscrBytes = TPR > 32 ? (TPR / 32) * 8 * kWarpBitmapWords<TPR> : 4;
+  // two-level rank: the product-loop chunk (one chunk of <= TPR A non-zeros) lives in the rank
+  // scratch (fine/pre2, unused until the gather), so the static shared memory stays small
   using BF = BlockFlat<VT, RANK2 ? flat_chunk_of<TPR>() : kFlatChunk>;
-  constexpr int kAuxBytes = TPR > 32 ? (kWscrBytes > (int)sizeof(BF) ? kWscrBytes : (int)sizeof(BF)) : 4;
+  static_assert(!RANK2 || sizeof(BF) <= (size_t)UPPER * 6, "chunk must fit the rank scratch");
+  constexpr int kAuxBytes = (TPR > 32 && !RANK2) ? (kWscrBytes > (int)sizeof(BF) ? kWscrBytes : (int)sizeof(BF)) : 16;
   __shared__ __align__(16) unsigned char s_aux[kAuxBytes];
   unsigned* s_wscr = reinterpret_cast<unsigned*>(s_aux);
   constexpr int NB = num_nbuckets(T);
@@ -570,14 +599,15 @@ __global__ __launch_bounds__(BS) void k_num_smem(NumArgs a) {
   const int row = active ? a.rows[ridx] : 0;
   if constexpr (RANK2) {
     static_assert(TPR == BS, "two-level rank: one row per CTA");
+    if (a.prof && threadIdx.x == 0) a.prof[4 * blockIdx.x + 1] = gtimer();
     Rank2 r2;
     r2.fine = reinterpret_cast<unsigned*>(Kp + T);
     r2.pre2 = reinterpret_cast<uint16_t*>(r2.fine + UPPER);
     r2.l1 = reinterpret_cast<unsigned*>(smem_raw + align16(T * (int)sizeof(VT) + T * 4 + (int)UPPER * 6));
     r2.p1 = r2.l1 + a.l1_words;
-    num_row<VT, TPR, false, true>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp,
+    num_row<VT, TPR, false, true, T, (int)(UPPER / TPR)>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp,
                                   reinterpret_cast<int*>(r2.fine), (uint16_t*)nullptr, T - 1, NB, s_lohi, ws, s_list,
-                                  &s_lcnt, s_wscr, reinterpret_cast<BF*>(s_aux), r2);
+                                  &s_lcnt, s_wscr, reinterpret_cast<BF*>(r2.fine), r2);
   } else {
     num_row<VT, TPR, false>(a, active, row, SKeys{smem_u32(Kp)}, SVals<VT>{smem_u32(Vp)}, Kp, Vp, Bc, S, T - 1, NB,
                             s_lohi + 2 * g, ws, s_list, &s_lcnt, s_wscr, reinterpret_cast<BF*>(s_aux));
@@ -626,12 +656,8 @@ cudaError_t launch_num_k(cudaStream_t s, const NumArgs& a, int smem) {
 
 // static shared memory of k_num_smem besides the dynamic tables
 template <typename VT, int TPR>
-constexpr int num_static_bytes() {
-  return 33 * 8 + 8 * 32 + 4 * kLongChunk + 16 +
-         (TPR > 32 ? (TPR / 32 * 8 * kWarpBitmapWords<TPR> > (int)sizeof(BlockFlat<VT, flat_chunk_of<TPR>()>)
-                          ? TPR / 32 * 8 * kWarpBitmapWords<TPR>
-                          : (int)sizeof(BlockFlat<VT, flat_chunk_of<TPR>()>))
-                   : 4);
+constexpr int num_static_bytes() {  // k_num_smem<..., RANK2 = true>
+  return 33 * 8 + 8 * 32 + 4 * kLongChunk + 16 + 16;
 }
 
 template <typename VT, int T, int TPR, int BS, long long UPPER>

@@ -13,6 +13,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -866,6 +867,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                          (long long)h->rbits.p, (long long)h->perm1.p};
     const bool ge = group_events(h);
     auto enqueue = [&]() -> spgemm_status_t {
+      if (ctotal > 0) CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
       CK(fork(h));
       for (int g = 0; g < kNumNumGroups; ++g) {
         const long long rows = (long long)h->snap2.num_rows[g];
@@ -893,9 +895,42 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
           gc.slab = static_cast<unsigned char*>(h->num_slab_c.p) + before * cstride;
           gc.bitmap_words = cwords;
           gc.slab_stride = cstride;
+          gc.row_counter = dacc->row_counter + c;
+          const char* pg = getenv("SPGEMM_PROF_GROUP");  // diagnostics: per-row phase timestamps
+          if (pg && atoi(pg) == g && !graphs_on(h)) {
+            CK(cudaMalloc(&gc.prof, sizeof(unsigned long long) * 4 * rows));
+            CK(cudaMemset(gc.prof, 0, sizeof(unsigned long long) * 4 * rows));
+          }
           CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
+          if (gc.prof) {
+            std::vector<unsigned long long> hp((size_t)(4 * rows));
+            CK(cudaStreamSynchronize(st));
+            CK(cudaMemcpy(hp.data(), gc.prof, hp.size() * 8, cudaMemcpyDeviceToHost));
+            cudaFree(gc.prof);
+            const char* out = getenv("SPGEMM_PROF_OUT");
+            if (FILE* f = fopen(out ? out : "spgemm_prof.bin", "wb")) {
+              fwrite(hp.data(), 8, hp.size(), f);
+              fclose(f);
+            }
+          }
         } else {
+          const char* pg = getenv("SPGEMM_PROF_GROUP");  // diagnostics: per-row phase timestamps
+          if (pg && atoi(pg) == g && !graphs_on(h)) {
+            CK(cudaMalloc(&ga.prof, sizeof(unsigned long long) * 4 * rows));
+            CK(cudaMemset(ga.prof, 0, sizeof(unsigned long long) * 4 * rows));
+          }
           CK(launch_numeric_group(st, g, fp64, ga));
+          if (ga.prof) {
+            std::vector<unsigned long long> hp((size_t)(4 * rows));
+            CK(cudaStreamSynchronize(st));
+            CK(cudaMemcpy(hp.data(), ga.prof, hp.size() * 8, cudaMemcpyDeviceToHost));
+            cudaFree(ga.prof);
+            const char* out = getenv("SPGEMM_PROF_OUT");
+            if (FILE* f = fopen(out ? out : "spgemm_prof.bin", "wb")) {
+              fwrite(hp.data(), 8, hp.size(), f);
+              fclose(f);
+            }
+          }
         }
         h->stats.kernel_launches_numeric += 1;
         if (ge) CK(cudaEventRecord(h->gstop[1][g], st));

@@ -114,6 +114,7 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   int b_unsorted;  // some B row is not strictly increasing (disables private accumulators)
   int cursor[2][kMaxGroups];
   int range_rmax;  // max column span R_i over the range rows (sizes the per-warp tables)
+  int row_counter[4];  // numeric cluster groups: dynamic row counters (zeroed per numeric call)
 };
 
 struct Bounds {  // group bounds passed by value
@@ -397,20 +398,39 @@ __device__ __forceinline__ void for_each_product_block(const int64_t* __restrict
     if (t < cn) sh->incl[t] = (int)(ex + len);
     __syncthreads();
     const int P = (int)tot;
+    // kU products per thread per round: all kU gathers are issued before any table update (B rows
+    // of graph shapes are short and scattered: each gather is an L2/HBM round trip)
+    constexpr int kU = 4;
 #pragma unroll 1
-    for (int p = t; p < P; p += tpr) {
-      int lo = 0, hi = cn - 1;  // first e with incl[e] > p
-      while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (sh->incl[mid] <= p) lo = mid + 1; else hi = mid;
+    for (int p0 = t; p0 < P; p0 += kU * tpr) {
+      int keys[kU];
+      VT vals[kU];
+      int es[kU];
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+        const int p = p0 + u * tpr;
+        es[u] = -1;
+        if (p < P) {
+          int lo = 0, hi = cn - 1;  // first e with incl[e] > p
+          while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (sh->incl[mid] <= p) lo = mid + 1; else hi = mid;
+          }
+          es[u] = lo;
+          const int start = lo ? sh->incl[lo - 1] : 0;
+          const long long q = sh->b0[lo] + (p - start);
+          keys[u] = __ldg(b_col + q);
+          vals[u] = NUM ? __ldg(b_val + q) : VT(0);
+        }
       }
-      const int e = lo;
-      const int start = e ? sh->incl[e - 1] : 0;
-      const long long q = sh->b0[e] + (p - start);
-      const int key = __ldg(b_col + q);
-      const VT v = NUM ? __ldg(b_val + q) : VT(0);
-      if (CHECK_STOP && stop()) break;
-      f(key, NUM ? sh->av[e] * v : VT(0));
+      bool stopped = false;
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+        if (es[u] < 0) continue;
+        if (CHECK_STOP && stop()) { stopped = true; break; }
+        f(keys[u], NUM ? sh->av[es[u]] * vals[u] : VT(0));
+      }
+      if (CHECK_STOP && stopped) break;
     }
     __syncthreads();
   }
@@ -724,7 +744,15 @@ struct NumArgs {
   void* slab; long long slab_T; long long slab_stride; long long max_nnz; long long bitmap_words;
   const unsigned* rbits; long long rwcap;  // range rows: symbolic pattern bitmap (same row order)
   int l1_words;            // CTA-per-row groups: level-1 words of the two-level rank (>= n/1024 + 1)
+  unsigned long long* prof;  // diagnostics (SPGEMM_PROF_GROUP): per CTA row, %globaltimer at phase ends
+  int* row_counter;          // cluster groups: dynamic row counter (zeroed by spgemm_numeric)
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
                                const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
