@@ -155,12 +155,12 @@ def load_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def load_traffic(phase, g):
+def load_traffic(phase, g, dtype):
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if not os.path.exists(p):
         return None
     d = json.load(open(p))
-    return d.get(f"{phase}_g{g}")
+    return d.get(f"{phase}_g{g}_{dtype}")
 
 
 # ----------------------------------------------------------------------------- reference arm
@@ -272,7 +272,7 @@ def run_ours(args):
     peak, peak_src = load_peaks()
     achieved = bytes_alg / (k_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": load_traffic(ph, g), "kernel": kernel_name(ph, g), "phase": ph, "group": g,
+                "traffic": load_traffic(ph, g, args.dtype), "kernel": kernel_name(ph, g), "phase": ph, "group": g,
                 "launch_ms": k_ms, "share_of_step": k_ms / (tot_ms / args.steps),
                 "algorithmic_bytes_per_launch": bytes_alg, "peak_source": peak_src}
 

@@ -43,6 +43,14 @@ def group_of(kname: str):
     if m:
         T, TPR, BS, up = int(m.group(2)), int(m.group(3)), int(m.group(4)), int(m.group(5))
         return "num", NUM.get((T, TPR, BS, up))
+    if re.search(r"k_sym_range(_bits)?\b", kname):
+        return "sym", 12  # kSymRange
+    if "k_num_range" in kname:
+        return "num", 14  # kNumRange
+    if "k_sym_cluster" in kname:
+        return "sym", 10
+    if "k_num_cluster" in kname:
+        return "num", 10
     return None, None
 
 
@@ -93,7 +101,8 @@ def full():
     uni = dict(zip(hdr, units))
     traffic = {}
     lines = [f"# ncu --set full ({TAG}) — group kernels of one bench step (cant-like A^2, fp32)", "",
-             "`ncu --set full --clock-control none --import-source on -k regex:\"k_(num|sym)_smem\" -c 4`", ""]
+             "`ncu --set full --clock-control none --import-source on -k regex:<group kernels> -c 6` "
+             "(scripts/gpu_round.sh)", ""]
     for r in rows[2:]:
         d = dict(zip(hdr, r))
         k = d["Kernel Name"]
@@ -115,7 +124,7 @@ def full():
         if ph:
             b = tobytes(d["dram__bytes_read.sum"], uni["dram__bytes_read.sum"]) + \
                 tobytes(d["dram__bytes_write.sum"], uni["dram__bytes_write.sum"])
-            traffic[f"{ph}_g{g}"] = int(b)
+            traffic[f"{ph}_g{g}_f32"] = int(b)  # the captured bench step is fp32
     open(os.path.join(OUT, f"ncu_{TAG}.md"), "w").write("\n".join(lines) + "\n")
     tj = os.path.join(OUT, "traffic.json")
     old = json.load(open(tj)) if os.path.exists(tj) else {}
