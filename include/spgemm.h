@@ -154,9 +154,16 @@ typedef enum {
                                        0: Table-I groups only.  Needs RANGE_HASH; off while a
                                        MIN_GROUP is forced */
     SPGEMM_OPT_RANGE_MIN_NPROD = 15,/* n_prod lower bound of range rows (default 256) */
-    SPGEMM_OPT_BITMAP_RANK = 16     /* 1 (default): CTA-per-row numeric groups order each row by a
+    SPGEMM_OPT_BITMAP_RANK = 16,    /* 1 (default): CTA-per-row numeric groups order each row by a
                                        two-level bitmap rank over its column span;
                                        0: bucket sort (ablation) */
+    SPGEMM_OPT_RANK_ACC = 17        /* 1 (default): CTA-per-row numeric groups (4-9) accumulate each
+                                       row directly at the rank of its column — the two-level
+                                       bitmap over the row's span built first, used as a
+                                       collision-free order-preserving hash;
+                                       needs RANGE_HASH (column spans).  0: paper hash table +
+                                       gather + rank; off while NUM_MIN_GROUP
+                                       is forced */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

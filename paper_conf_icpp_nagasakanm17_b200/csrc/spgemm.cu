@@ -85,6 +85,7 @@ struct spgemm_ctx {
   int timing = 1;
   int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
   long long range_min_np = kRangeMinNprodDefault;
+  int rank_acc = 1;      // CTA-per-row numeric groups: rank-indexed accumulation (kernels_rankacc.cu)
   int bitmap_rank = 1;   // CTA-per-row numeric groups: two-level bitmap rank (else bucket sort)
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -507,6 +508,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       if (v < 1 || v > kRangeMaxNprod) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_MIN_NPROD out of range");
       h->range_min_np = v; break;
     case SPGEMM_OPT_BITMAP_RANK: h->bitmap_rank = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_ACC: h->rank_acc = v ? 1 : 0; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -827,6 +829,13 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.priv_ok = h->snap1.b_unsorted ? 0 : 1;
     na.err_flags = &dacc->err_flags;
     na.l1_words = h->bitmap_rank ? (int)((h->n + 1023) / 1024 + 1) : 0;
+    // rank-indexed accumulation for the CTA-per-row groups (needs the column spans; the forced
+    // paths keep the paper hash)
+    const int l1w_rank = (int)((h->n + 1023) / 1024 + 1);
+    auto rank_acc_on = [&](int g) {
+      return h->rank_acc && h->rlohi.p != nullptr && h->num_min_group < 0 && g >= 4 && g <= 9 &&
+             rankacc_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit;
+    };
     // cluster groups (clusters of 2/4/8 CTAs): bitmap + prefix scratch per resident cluster
     const long long cwords = h->n / 32 + 2;
     const long long cstride = (2 * cwords * 4 + 255) & ~255LL;
@@ -858,7 +867,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // numeric re-runs with new values of the same structure, or repeated multiplies)
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
-                                   h->snap1.range_rmax, (long long)na.l1_words};
+                                   h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
@@ -919,7 +928,13 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(cudaMalloc(&ga.prof, sizeof(unsigned long long) * 4 * rows));
             CK(cudaMemset(ga.prof, 0, sizeof(unsigned long long) * 4 * rows));
           }
-          CK(launch_numeric_group(st, g, fp64, ga));
+          if (rank_acc_on(g)) {
+            NumArgs ra = ga;
+            ra.l1_words = l1w_rank;
+            CK(launch_numeric_rankacc(st, g, fp64, ra));
+          } else {
+            CK(launch_numeric_group(st, g, fp64, ga));
+          }
           if (ga.prof) {
             std::vector<unsigned long long> hp((size_t)(4 * rows));
             CK(cudaStreamSynchronize(st));

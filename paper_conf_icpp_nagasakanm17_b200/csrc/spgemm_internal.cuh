@@ -776,6 +776,8 @@ cudaError_t launch_symbolic_group(cudaStream_t s, int group, const SymArgs& a, i
 cudaError_t launch_symbolic_global(cudaStream_t s, const SymArgs& a, int grid);
 cudaError_t launch_numeric_group(cudaStream_t s, int group, bool fp64, const NumArgs& a);
 cudaError_t launch_numeric_global(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
+cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const NumArgs& a);
+int rankacc_smem_bytes(int group, bool fp64, int l1_words);
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows);
 cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);

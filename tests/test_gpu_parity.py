@@ -533,3 +533,50 @@ def test_rmat_s22_sampled(spg):
         starts[C.rpt[1:-1][C.rpt[1:-1] < C.nnz]] = True
         assert bool(((d > 0) | starts[1:]).all())
         assert st["nnz_c"] == C.nnz
+
+
+# ------------------------------------------------------------------ rank-indexed accumulation
+# CTA-per-row numeric groups 4-9 accumulate at the rank of the column from a two-level bitmap of
+# the row's span (kernels_rankacc.cu).  Fast path: <= TPR A non-zeros and
+# <= 8*TPR products held in registers; slow path: chunked re-walks (QCD-like rows: 1521 products,
+# 210 outputs, so products > 8*TPR in group 4).
+
+def _rank_rows(st):
+    return sum(st["num_rows"][g] for g in range(4, 10))
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("name", ["rmat14", "webbase_small", "mixed:qcd", "mixed:circuit"])
+def test_rank_acc_vs_paper_hash(spg, name, dtype):
+    A = _mixed_small() if name == "webbase_small" else (
+        synth.rmat(14).with_values("uniform", 9) if name == "rmat14" else synth.config(name))
+    got = check(spg, A, A, dtype, what=f"{name} rank_acc")
+    if name != "mixed:circuit":
+        assert _rank_rows(got[3]) > 0, "no rows in the rank-accumulate groups"
+    check(spg, A, A, dtype, opts={"rank_acc": 0}, what=f"{name} paper hash")
+
+
+@pytest.mark.parametrize("name", ["rmat14", "mixed:qcd"])
+def test_rank_acc_int_exact(spg, name):
+    A = synth.rmat(14).with_values("int", 2) if name == "rmat14" else synth.config(name, "int")
+    check(spg, A, A, np.float32, exact=True, what=f"{name} int")
+
+
+def test_rank_acc_duplicates_and_unsorted(spg):
+    # duplicate and unsorted columns inside B rows: equal keys share one rank (summed)
+    rng = np.random.default_rng(21)
+    m = 1500
+    rows = np.repeat(np.arange(m), 200)
+    cols = rng.integers(0, 200000, size=rows.size)
+    dup = rng.random(rows.size) < 0.2
+    cols[dup] = cols[np.maximum(np.arange(rows.size) - 1, 0)][dup]
+    A = from_coo(m, 200000, rows, cols, rng.uniform(-1, 1, rows.size), dedup=False)
+    B = from_coo(200000, 200000, rng.integers(0, 200000, 800000), rng.integers(0, 200000, 800000),
+                 rng.uniform(-1, 1, 800000), dedup=False)
+    for M in (A, B):  # shuffle the entries inside every row
+        r = np.repeat(np.arange(M.m), np.diff(M.rpt))
+        o = np.lexsort((rng.random(r.size), r))
+        M.col[:] = M.col[o]
+        M.val[:] = M.val[o]
+    got = check(spg, A, B, np.float64, what="dup/unsorted rank_acc")
+    assert _rank_rows(got[3]) > 0
