@@ -1,32 +1,38 @@
-// kernels_rankacc.cu — numeric step (7) for CTA-per-row groups of wide-span (graph) rows:
-// accumulation into a table indexed by the RANK of the column in the row (B200 addition,
-// DESIGN.md §5.8).
+// kernels_rankacc.cu — CTA-per-row kernels for wide-span (graph) rows that index the row's
+// table by the RANK of the column (B200 addition): symbolic count (step 3) and
+// numeric accumulate + gather + sort (step 7).
 //
 // The paper's numeric phase inserts every product's column into a hash table
 // (Alg. 5), adds the value into a parallel value table, then gathers the occupied slots and sorts
-// them by a comparison rank.  Its final position is rank(key) = #distinct columns of row i below
-// key.  For rows of C whose column span is wide and sparse (power-law graphs: R-MAT, webbase —
-// products ~ output entries, so the hash tables are nearly all fixed cost) this kernel computes
+// them by a comparison rank; the symbolic phase counts the distinct keys of the same table
+// (PAPER.md:130-155).  An entry's final position is rank(key) = #distinct columns of row i below
+// key.  For rows whose column span is wide and sparse (power-law graphs: R-MAT, webbase — products
+// ~ output entries, so the 2x-oversized hash tables are nearly all fixed cost) these kernels build
 // that rank FIRST, from a two-level bitmap of the row's columns over its exact span [lo_i, hi_i]
-// (from step (1)), and uses it as a collision-free, order-preserving hash:
+// (computed with n_prod in step (1)), and use it as a collision-free, order-preserving hash:
 //
-//   (i)   metadata: the row's A non-zeros (<= TPR), one per thread: col_A, val_A, rpt_B pair;
-//         block scan of the B-row lengths (Alg. 3/4's product enumeration, flattened);
+//   (i)   metadata: the row's A non-zeros (<= MC*TPR), MC consecutive ones per thread: col_A,
+//         val_A, rpt_B pair; block scan of the B-row lengths (Alg. 3/4's product enumeration,
+//         flattened) and, per 32-product block, the A entry holding its first product (a product
+//         finds its entry with one lookup and a short forward walk instead of a binary search);
 //   (ii)  gather: thread t takes products t, t+TPR, ... (<= KP of them, held in registers; all
-//         gathers of b_col/b_val issued before use) and sets level-1 bit (key-lo)>>5 — "32-column
-//         block is non-empty" — with a shared atomicOr;
+//         gathers of b_col/b_val issued before use) and sets level-1 bit (key-lo)>>5 — "this
+//         32-column block is non-empty" — with a shared atomicOr;
 //   (iii) prefix popcount of level 1 -> compact index of every non-empty block;
 //   (iv)  each product sets its bit in the level-2 word of its block;
+//   symbolic: nnz_i = popcount of level 2 (the count of inserted keys).
+//   numeric:
 //   (v)   prefix popcount of level 2 -> rank(key) = pre2[b] + popc(fine[b] & below(key));
 //   (vi)  vals[rank] += a_ik * b_kj (shared atomic add, working precision),
 //         keys[rank] = key (idempotent store);
-//   (vii) the row is now compact and sorted: coalesced write of keys/vals to C.
+//   (vii) the row is compact and sorted: coalesced write of keys/vals to C.
 //
 // No probing, no -1 initialisation of a 2x-oversized table, no compaction or sort pass; O(n_prod
-// + R_i/1024) work with a handful of CTA barriers.  Rows with more than TPR A non-zeros or more
-// than KP*TPR products walk the products with the chunked block loop once per pass (re-gathering;
-// the result is identical).  The paper's hash path (kernels_numeric.cu) stays for rows without a
-// column span (range hash disabled) and as the forced-path reference.
+// + R_i/1024) work per row.  Rows with more than MC*TPR A non-zeros or more than KP*TPR products
+// walk their products with the chunked block loop once per pass (re-gathering; identical result).
+// The paper's hash kernels (kernels_symbolic.cu, kernels_numeric.cu) remain for rows without a
+// column span (range hash disabled), for the forced-group paths and as the ablation
+// (SPGEMM_OPT_RANK_ACC = 0).
 #include <climits>
 
 #include "spgemm_internal.cuh"
@@ -64,81 +70,136 @@ __device__ __forceinline__ int cta_scan32(int v, int* total, int* ws32) {
   return (w > 0 ? base : 0) + x - v;
 }
 
-// Dynamic shared memory layout (16-byte aligned pieces):
-//   vals[UPPER] VT | b0[TPR] i64 | av[TPR] VT | incl[TPR] i32 | keys[UPPER] i32 |
-//   fine[UPPER] u32 | l1[L1W] u32 | pre2[UPPER] u16 | p1[L1W] u16
-template <typename VT, int TPR, long long UPPER>
+__device__ __forceinline__ int popc4(uint4 x) { return __popc(x.x) + __popc(x.y) + __popc(x.z) + __popc(x.w); }
+
+// Exclusive prefix popcount of words[0..W) (W rounded up to 4 words, the tail zero) into pre
+// (u16, may be null); returns the total.  One contiguous run of uint4 per thread.
+template <int TPR>
+__device__ __forceinline__ int prefix_popc(const unsigned* words, int W, uint16_t* pre, int* ws32) {
+  const int W4 = (W + 3) >> 2;
+  const int per = (W4 + TPR - 1) / TPR;
+  const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
+  const uint4* w4 = reinterpret_cast<const uint4*>(words);
+  int loc = 0;
+  for (int v = v0; v < v1; ++v) loc += popc4(w4[v]);
+  int total;
+  int run = cta_scan32<TPR>(loc, &total, ws32);
+  if (pre) {
+    for (int v = v0; v < v1; ++v) {
+      const uint4 x = w4[v];
+      ushort4 o;
+      o.x = (unsigned short)run; run += __popc(x.x);
+      o.y = (unsigned short)run; run += __popc(x.y);
+      o.z = (unsigned short)run; run += __popc(x.z);
+      o.w = (unsigned short)run; run += __popc(x.w);
+      reinterpret_cast<ushort4*>(pre)[v] = o;
+    }
+  }
+  return total;
+}
+
+template <int TPR>
+__device__ __forceinline__ void clear_words(unsigned* words, int W) {
+  uint4* w4 = reinterpret_cast<uint4*>(words);
+  for (int v = threadIdx.x; v < (W + 3) >> 2; v += TPR) w4[v] = make_uint4(0u, 0u, 0u, 0u);
+}
+
+// Shared-memory layout of one row (16-byte aligned pieces); VT = value type (int: symbolic).
+//   vals[UPPER] VT (numeric) | b0[ME] i64 | av[ME] VT (numeric) | incl[ME] i32 |
+//   keys[UPPER] i32 (numeric) | fine[UPPER] u32 | bstart[KP*TPR/32+1] i32 | l1[L1W] u32 |
+//   pre2[UPPER] u16 (numeric) | p1[L1W] u16
+template <typename VT, bool NUM, int TPR, long long UPPER, int MC, int KP>
 struct RankLayout {
+  static constexpr int ME = MC * TPR;  // metadata entries
   static constexpr int kVals = 0;
-  static constexpr int kB0 = align16((int)(UPPER * sizeof(VT)));
-  static constexpr int kAv = kB0 + align16(TPR * 8);
-  static constexpr int kIncl = kAv + align16(TPR * (int)sizeof(VT));
-  static constexpr int kKeys = kIncl + align16(TPR * 4);
-  static constexpr int kFine = kKeys + align16((int)UPPER * 4);
-  static constexpr int kL1 = kFine + align16((int)UPPER * 4);
+  static constexpr int kB0 = NUM ? align16((int)(UPPER * sizeof(VT))) : 0;
+  static constexpr int kAv = kB0 + align16(ME * 8);
+  static constexpr int kIncl = kAv + (NUM ? align16(ME * (int)sizeof(VT)) : 0);
+  static constexpr int kKeys = kIncl + align16(ME * 4);
+  static constexpr int kFine = kKeys + (NUM ? align16((int)UPPER * 4) : 0);
+  static constexpr int kBstart = kFine + align16((int)UPPER * 4);
+  static constexpr int kL1 = kBstart + align16((KP * TPR / 32 + 1) * 4);
   static __host__ __device__ constexpr int pre2(int l1w) { return kL1 + align16(l1w * 4); }
-  static __host__ __device__ constexpr int p1(int l1w) { return pre2(l1w) + align16((int)UPPER * 2); }
+  static __host__ __device__ constexpr int p1(int l1w) { return pre2(l1w) + (NUM ? align16((int)UPPER * 2) : 0); }
   static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1w * 2); }
 };
 
-template <typename VT, int TPR, long long UPPER, int KP>
-__global__ __launch_bounds__(TPR, TPR >= 1024 ? 1 : 2048 / TPR / 2) void k_num_rankacc(NumArgs a) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  using L = RankLayout<VT, TPR, UPPER>;
-  __shared__ int ws32[2][32];
-  __shared__ long long ws64[33];
+constexpr int kMetaPerThread = 2;
+__host__ __device__ constexpr int rankbig_l1pad_h(int l1w) { return (l1w + 3) & ~3; }  // MC: A non-zeros of a row held as metadata per thread
+
+// Adapters so rank_row reads both argument structs the same way.
+struct NumView : NumArgs {
+  __device__ __forceinline__ const void* a_val_ptr() const { return a_val; }
+  __device__ __forceinline__ const void* b_val_ptr() const { return b_val; }
+};
+struct SymView : SymArgs {
+  __device__ __forceinline__ const void* a_val_ptr() const { return nullptr; }
+  __device__ __forceinline__ const void* b_val_ptr() const { return nullptr; }
+};
+
+// One row, symbolic (NUM = false: writes nnz_i to c_cnt[row]) or numeric (writes the row of C).
+template <typename VT, bool NUM, int TPR, long long UPPER, int KP, typename Args>
+__device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* smem_raw, int (*ws32)[32],
+                                         long long* ws64) {
+  constexpr int MC = kMetaPerThread;
+  using L = RankLayout<VT, NUM, TPR, UPPER, MC, KP>;
+  constexpr int ME = L::ME;
   VT* vals = reinterpret_cast<VT*>(smem_raw + L::kVals);
   long long* sb0 = reinterpret_cast<long long*>(smem_raw + L::kB0);
   VT* sav = reinterpret_cast<VT*>(smem_raw + L::kAv);
   int* sincl = reinterpret_cast<int*>(smem_raw + L::kIncl);
   int* keys = reinterpret_cast<int*>(smem_raw + L::kKeys);
   unsigned* fine = reinterpret_cast<unsigned*>(smem_raw + L::kFine);
+  int* bstart = reinterpret_cast<int*>(smem_raw + L::kBstart);
   unsigned* l1 = reinterpret_cast<unsigned*>(smem_raw + L::kL1);
   uint16_t* pre2 = reinterpret_cast<uint16_t*>(smem_raw + L::pre2(a.l1_words));
   uint16_t* p1 = reinterpret_cast<uint16_t*>(smem_raw + L::p1(a.l1_words));
-  // the chunked fallback walk reuses b0/av/incl through the BlockFlat view (same field order)
-  static_assert(sizeof(BlockFlat<VT, TPR>) <= (size_t)(L::kKeys - L::kB0) + 64, "block-flat view");
 
-  const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val);
-  const VT* __restrict__ bv_g = static_cast<const VT*>(a.b_val);
+  const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val_ptr());
+  const VT* __restrict__ bv_g = static_cast<const VT*>(a.b_val_ptr());
   const int32_t* __restrict__ bc_g = a.b_col;
   const int t = threadIdx.x;
-  const int row = a.rows[blockIdx.x];
   const long long a0 = __ldg(a.a_rpt + row);
   const int na = (int)(__ldg(a.a_rpt + row + 1) - a0);
-  const long long c0 = a.c_rpt[row];
-  const int cn = (int)(a.c_rpt[row + 1] - c0);
   const int2 rr = __ldg(a.rlohi + row);
   const int lo = rr.x;
   const int W1 = rr.y >= rr.x ? (int)(((unsigned)(rr.y - rr.x)) >> 10) + 1 : 0;  // CTA-uniform
-  for (int w = t; w < W1; w += TPR) l1[w] = 0u;
+  clear_words<TPR>(l1, W1);
 
-  // (i) metadata of the first TPR A non-zeros + scan of their B-row lengths
-  int len = 0;
-  if (t < na) {
-    const int kk = __ldg(a.a_col + a0 + t);
-    const long long b0 = __ldg(a.b_rpt + kk);
-    len = (int)(__ldg(a.b_rpt + kk + 1) - b0);
-    sb0[t] = b0;
-    sav[t] = __ldg(av_g + a0 + t);
+  // (i) metadata: thread t owns A non-zeros t*MC .. t*MC+MC-1
+  int lens[MC];
+  int mysum = 0;
+#pragma unroll
+  for (int j = 0; j < MC; ++j) {
+    const int e = t * MC + j;
+    lens[j] = 0;
+    if (e < na) {
+      const int kk = __ldg(a.a_col + a0 + e);
+      const long long b0 = __ldg(a.b_rpt + kk);
+      lens[j] = (int)(__ldg(a.b_rpt + kk + 1) - b0);
+      sb0[e] = b0;
+      if constexpr (NUM) sav[e] = __ldg(av_g + a0 + e);
+    }
+    mysum += lens[j];
   }
   int P;
-  const int ex = cta_scan32<TPR>(t < na ? len : 0, &P, ws32[0]);
-  if (t < na) sincl[t] = ex + len;
+  int run = cta_scan32<TPR>(mysum, &P, ws32[0]);
+  const bool fast = na <= ME && P <= KP * TPR;  // CTA-uniform
+#pragma unroll
+  for (int j = 0; j < MC; ++j) {
+    const int e = t * MC + j;
+    if (e < na) {
+      const int s = run, en = run + lens[j];
+      sincl[e] = en;
+      if (fast)  // 32-product blocks whose first product lies in this entry
+        for (int k = (s + 31) >> 5; k < ((en + 31) >> 5); ++k) bstart[k] = e;
+      run = en;
+    }
+  }
   __syncthreads();
-  const bool fast = na <= TPR && P <= KP * TPR;  // CTA-uniform
 
   int key[KP];
   VT val[KP];
-  auto locate = [&](int p, int& e, long long& q) {  // product p -> its A entry e and B position q
-    int l = 0, h = min(na, TPR) - 1;
-    while (l < h) {
-      const int mid = (l + h) >> 1;
-      if (sincl[mid] <= p) l = mid + 1; else h = mid;
-    }
-    e = l;
-    q = sb0[l] + (p - (l ? sincl[l - 1] : 0));
-  };
   auto set_l1 = [&](int k) {
     const unsigned d = (unsigned)(k - lo);
     atomicOr(l1 + (d >> 10), 1u << ((d >> 5) & 31));
@@ -159,9 +220,10 @@ __global__ __launch_bounds__(TPR, TPR >= 1024 ? 1 : 2048 / TPR / 2) void k_num_r
     keys[r] = k;
   };
   BlockFlat<VT, TPR>* bf = reinterpret_cast<BlockFlat<VT, TPR>*>(sb0);
+  static_assert(sizeof(BlockFlat<VT, TPR>) <= (size_t)(L::kKeys - L::kB0) + 16, "block-flat view");
   auto walk = [&](auto&& f) {  // slow path: chunked block loop over all products (re-gathers)
-    for_each_product_block<true, false, VT, TPR>(a.a_rpt, a.a_col, av_g, a.b_rpt, bc_g, bv_g, true, row, t, bf,
-                                                 ws64, f, NoStopR{});
+    for_each_product_block<NUM, false, VT, TPR>(a.a_rpt, a.a_col, av_g, a.b_rpt, bc_g, bv_g, true, row, t, bf, ws64,
+                                                f, NoStopR{});
   };
 
   // (ii) gather + level 1
@@ -171,111 +233,289 @@ __global__ __launch_bounds__(TPR, TPR >= 1024 ? 1 : 2048 / TPR / 2) void k_num_r
       const int p = t + u * TPR;
       key[u] = -1;
       if (p < P) {
-        int e;
-        long long q;
-        locate(p, e, q);
+        int e = bstart[p >> 5];
+        while (sincl[e] <= p) ++e;
+        const long long q = sb0[e] + (p - (e ? sincl[e - 1] : 0));
         key[u] = __ldg(bc_g + q);
-        val[u] = sav[e] * __ldg(bv_g + q);
+        if constexpr (NUM) val[u] = sav[e] * __ldg(bv_g + q);
       }
     }
 #pragma unroll
     for (int u = 0; u < KP; ++u)
       if (key[u] >= 0) set_l1(key[u]);
   } else {
-    __syncthreads();  // the walk overwrites b0/av/incl
     walk([&](int k, VT) { set_l1(k); });
   }
   __syncthreads();
   // (iii) compact index of the non-empty 32-column blocks
-  int nb;
-  {
-    const int per = (W1 + TPR - 1) / TPR;
-    const int w0 = min(W1, t * per), w1 = min(W1, w0 + per);
-    int loc = 0;
-    for (int w = w0; w < w1; ++w) loc += __popc(l1[w]);
-    int run = cta_scan32<TPR>(loc, &nb, ws32[1]);
-    for (int w = w0; w < w1; ++w) { p1[w] = (uint16_t)run; run += __popc(l1[w]); }
-  }
-  for (int b = t; b < nb; b += TPR) fine[b] = 0u;
+  const int nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
+  const bool ok = nb <= (int)UPPER;  // CTA-uniform; false only for inconsistent input
+  if (ok) clear_words<TPR>(fine, nb);
   __syncthreads();
   // (iv) level 2
-  if (fast) {
+  if (ok) {
+    if (fast) {
 #pragma unroll
-    for (int u = 0; u < KP; ++u)
-      if (key[u] >= 0) set_fine(key[u]);
+      for (int u = 0; u < KP; ++u)
+        if (key[u] >= 0) set_fine(key[u]);
+    } else {
+      walk([&](int k, VT) { set_fine(k); });
+    }
+  }
+  __syncthreads();
+  if constexpr (!NUM) {
+    // symbolic: nnz_i = number of distinct columns = popcount of level 2
+    const int n = ok ? prefix_popc<TPR>(fine, nb, nullptr, ws32[0]) : 0;
+    if (t == 0) {
+      a.c_cnt[row] = n;
+      if (!ok) atomicOr(a.err_flags, 1);
+    }
   } else {
-    walk([&](int k, VT) { set_fine(k); });
-  }
-  __syncthreads();
-  // (v) rank of every block's first key
-  int n_total;
-  {
-    const int per = (nb + TPR - 1) / TPR;
-    const int b0 = min(nb, t * per), b1 = min(nb, b0 + per);
-    int loc = 0;
-    for (int b = b0; b < b1; ++b) loc += __popc(fine[b]);
-    int run = cta_scan32<TPR>(loc, &n_total, ws32[0]);
-    for (int b = b0; b < b1; ++b) { pre2[b] = (uint16_t)run; run += __popc(fine[b]); }
-  }
-  if (t == 0 && n_total != cn) atomicOr(a.err_flags, 2);
-  const int nw = min(n_total, cn);
-  for (int r = t; r < nw; r += TPR) vals[r] = VT(0);
-  __syncthreads();
-  // (vi) accumulate at the rank
-  if (fast) {
+    const long long c0 = a.c_rpt[row];
+    const int cn = (int)(a.c_rpt[row + 1] - c0);
+    // (v) rank of every block's first key
+    const int n_total = ok ? prefix_popc<TPR>(fine, nb, pre2, ws32[0]) : 0;
+    if (t == 0 && n_total != cn) atomicOr(a.err_flags, 2);
+    const int nw = ok ? min(n_total, cn) : 0;
+    for (int r = t; r < nw; r += TPR) vals[r] = VT(0);
+    __syncthreads();
+    // (vi) accumulate at the rank
+    if (ok) {
+      if (fast) {
 #pragma unroll
-    for (int u = 0; u < KP; ++u)
-      if (key[u] >= 0) accumulate(key[u], val[u]);
-  } else {
-    walk([&](int k, VT v) { accumulate(k, v); });
+        for (int u = 0; u < KP; ++u)
+          if (key[u] >= 0) accumulate(key[u], val[u]);
+      } else {
+        walk([&](int k, VT v) { accumulate(k, v); });
+      }
+    }
+    __syncthreads();
+    // (vii) sorted, compact row -> C (coalesced)
+    int32_t* __restrict__ cc = a.c_col + c0;
+    VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+    for (int r = t; r < nw; r += TPR) {
+      cc[r] = keys[r];
+      cv[r] = vals[r];
+    }
   }
-  __syncthreads();
-  // (vii) sorted, compact row -> C (coalesced)
-  int32_t* __restrict__ cc = a.c_col + c0;
-  VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
-  for (int r = t; r < nw; r += TPR) {
-    cc[r] = keys[r];
-    cv[r] = vals[r];
+}
+
+template <typename VT>
+constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 4 + (int)sizeof(BlockFlat<VT, 1024>); }
+
+// 40 registers (1536 threads per SM) for fp32 / symbolic; fp64 values need 64 (no spills)
+template <int TPR, int VB>
+constexpr int rank_min_blocks() { return TPR >= 1024 ? 1 : (VB > 4 ? 1024 : 1536) / TPR; }
+
+template <typename VT, int TPR, long long UPPER, int KP>
+__global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT)>()) void k_num_rankacc(NumArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ int ws32[2][32];
+  __shared__ long long ws64[33];
+  rank_row<VT, true, TPR, UPPER, KP>(static_cast<const NumView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
+}
+
+template <int TPR, long long UPPER, int KP>
+__global__ __launch_bounds__(TPR, rank_min_blocks<TPR, 4>()) void k_sym_rankcnt(SymArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ int ws32[2][32];
+  __shared__ long long ws64[33];
+  rank_row<int, false, TPR, UPPER, KP>(static_cast<const SymView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
+}
+
+constexpr int kNumKP = 8;
+template <int TPR, long long UPPER>
+constexpr int sym_kp() { return (int)(UPPER / TPR) > 16 ? 16 : (int)(UPPER / TPR); }
+
+template <typename K>
+cudaError_t prepare(K kernel, int smem, int& configured) {
+  if (smem > configured) {
+    cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    // the rows' B gathers are scattered (L1 hit rates ~30%): give the SM's memory to the tables
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+    configured = smem;
   }
+  return cudaSuccess;
 }
 
 template <typename VT, int TPR, long long UPPER>
 cudaError_t launch_rankacc_k(cudaStream_t s, const NumArgs& a) {
-  constexpr int KP = 8;
-  using L = RankLayout<VT, TPR, UPPER>;
+  using L = RankLayout<VT, true, TPR, UPPER, kMetaPerThread, kNumKP>;
   const int smem = L::bytes(a.l1_words);
   static int configured = 0;
-  if (smem > configured) {
-    cudaError_t e = cudaFuncSetAttribute(k_num_rankacc<VT, TPR, UPPER, KP>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    configured = smem;
-  }
-  k_num_rankacc<VT, TPR, UPPER, KP><<<(unsigned)a.nrows, TPR, smem, s>>>(a);
+  cudaError_t e = prepare(k_num_rankacc<VT, TPR, UPPER, kNumKP>, smem, configured);
+  if (e != cudaSuccess) return e;
+  k_num_rankacc<VT, TPR, UPPER, kNumKP><<<(unsigned)a.nrows, TPR, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+template <int TPR, long long UPPER>
+cudaError_t launch_rankcnt_k(cudaStream_t s, const SymArgs& a) {
+  constexpr int KP = sym_kp<TPR, UPPER>();
+  using L = RankLayout<int, false, TPR, UPPER, kMetaPerThread, KP>;
+  const int smem = L::bytes(a.l1_words);
+  static int configured = 0;
+  cudaError_t e = prepare(k_sym_rankcnt<TPR, UPPER, KP>, smem, configured);
+  if (e != cudaSuccess) return e;
+  k_sym_rankcnt<TPR, UPPER, KP><<<(unsigned)a.nrows, TPR, smem, s>>>(a);
   return cudaGetLastError();
 }
 
 template <typename VT>
 cudaError_t launch_rankacc_v(cudaStream_t s, int group, const NumArgs& a) {
   switch (group) {
-#define SPG_G(I)                                                                                  \
-  case I:                                                                                         \
-    return launch_rankacc_k<VT, kNumGroups[I].TPR, kNumGroups[I].upper>(s, a);
+#define SPG_G(I) \
+  case I: return launch_rankacc_k<VT, kNumGroups[I].TPR, kNumGroups[I].upper>(s, a);
     SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return cudaErrorInvalidValue;
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// Rows above the largest CTA group (nnz_i > 8192; numeric groups 10-12): one 1024-thread CTA per
+// row, persistent, rows handed out through a global counter.  Level 1 (and its u32 prefix) stays
+// in shared memory; level 2 and its prefix live in a per-CTA global slab (L2-resident; up to
+// 8 B per output entry); values are accumulated directly into the row of C at their rank
+// (red.global.add, working precision) after the row is zeroed, keys stored there too.  Products
+// are walked three times (level 1, level 2, accumulate) with the chunked block loop; the second
+// and third walks re-gather B rows that the first one brought into L2.
+template <int TPR>
+__device__ __forceinline__ int prefix_popc32(const unsigned* words, int W, unsigned* pre, int* ws32, bool global) {
+  const int W4 = (W + 3) >> 2;
+  const int per = (W4 + TPR - 1) / TPR;
+  const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
+  const uint4* w4 = reinterpret_cast<const uint4*>(words);
+  auto ld = [&](int v) { return global ? __ldcg(w4 + v) : w4[v]; };
+  int loc = 0;
+  for (int v = v0; v < v1; ++v) loc += popc4(ld(v));
+  int total;
+  int run = cta_scan32<TPR>(loc, &total, ws32);
+  for (int v = v0; v < v1; ++v) {
+    const uint4 x = ld(v);
+    uint4 o;
+    o.x = (unsigned)run; run += __popc(x.x);
+    o.y = (unsigned)run; run += __popc(x.y);
+    o.z = (unsigned)run; run += __popc(x.z);
+    o.w = (unsigned)run; run += __popc(x.w);
+    reinterpret_cast<uint4*>(pre)[v] = o;
+  }
+  return total;
+}
+
+
+template <typename VT>
+__global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
+  constexpr int TPR = 1024;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ int ws32[2][32];
+  __shared__ long long ws64[33];
+  __shared__ int s_i;
+  const int l1p = rankbig_l1pad_h(a.l1_words);
+  unsigned* l1 = reinterpret_cast<unsigned*>(smem_raw);
+  unsigned* p1 = l1 + l1p;
+  BlockFlat<VT, TPR>* bf = reinterpret_cast<BlockFlat<VT, TPR>*>(p1 + l1p);
+  unsigned* fine = reinterpret_cast<unsigned*>(static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride);
+  unsigned* pre2 = fine + a.slab_T;
+  const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val);
+  const VT* __restrict__ bv_g = static_cast<const VT*>(a.b_val);
+  const int t = threadIdx.x;
+  while (true) {
+    if (t == 0) s_i = atomicAdd(a.row_counter, 1);
+    __syncthreads();
+    const int i = s_i;
+    if (i >= a.nrows) break;  // CTA-uniform
+    const int row = a.rows[i];
+    const int2 rr = __ldg(a.rlohi + row);
+    const int lo = rr.x;
+    const int W1 = rr.y >= rr.x ? (int)(((unsigned)(rr.y - rr.x)) >> 10) + 1 : 0;
+    const long long c0 = a.c_rpt[row];
+    const int cn = (int)(a.c_rpt[row + 1] - c0);
+    int32_t* __restrict__ cc = a.c_col + c0;
+    VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+    clear_words<TPR>(l1, W1);
+    for (int r = t; r < cn; r += TPR) cv[r] = VT(0);
+    auto walk = [&](auto&& f) {
+      for_each_product_block<true, false, VT, TPR>(a.a_rpt, a.a_col, av_g, a.b_rpt, a.b_col, bv_g, true, row, t, bf,
+                                                   ws64, f, NoStopR{});
+    };
+    auto blk_of = [&](unsigned d) {
+      const unsigned w = d >> 10, bit = (d >> 5) & 31;
+      return (int)p1[w] + __popc(l1[w] & ((1u << bit) - 1u));
+    };
+    __syncthreads();
+    walk([&](int k, VT) {
+      const unsigned d = (unsigned)(k - lo);
+      atomicOr(l1 + (d >> 10), 1u << ((d >> 5) & 31));
+    });
+    __syncthreads();
+    const int nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
+    const bool ok = nb <= (int)a.slab_T;  // CTA-uniform; false only for inconsistent input
+    if (ok) {
+      uint4* f4 = reinterpret_cast<uint4*>(fine);
+      for (int v = t; v < (nb + 3) >> 2; v += TPR) f4[v] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    __syncthreads();
+    if (ok)
+      walk([&](int k, VT) {
+        const unsigned d = (unsigned)(k - lo);
+        atomicOr(fine + blk_of(d), 1u << (d & 31));
+      });
+    __syncthreads();
+    const int n_total = ok ? prefix_popc32<TPR>(fine, nb, pre2, ws32[0], true) : 0;
+    if (t == 0 && n_total != cn) atomicOr(a.err_flags, 2);
+    __syncthreads();
+    if (ok && n_total == cn)
+      walk([&](int k, VT v) {
+        const unsigned d = (unsigned)(k - lo);
+        const int b = blk_of(d);
+        const int r = (int)__ldcg(pre2 + b) + __popc(__ldcg(fine + b) & ((1u << (d & 31)) - 1u));
+        atomicAdd(cv + r, v);
+        cc[r] = k;
+      });
+    __syncthreads();
+  }
+}
+
+template <typename VT>
+cudaError_t launch_rankbig_v(cudaStream_t s, const NumArgs& a, int grid) {
+  const int smem = rankbig_smem_bytes_v<VT>(a.l1_words);
+  static int configured = 0;
+  cudaError_t e = prepare(k_num_rankbig<VT>, smem, configured);
+  if (e != cudaSuccess) return e;
+  k_num_rankbig<VT><<<grid, 1024, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+constexpr int kStaticRankBytes = 2 * 32 * 4 + 33 * 8 + 1024;  // static shared + driver reserve
+
 }  // namespace
 
 int rankacc_smem_bytes(int group, bool fp64, int l1_words) {
   switch (group) {
-#define SPG_G(I)                                                                                              \
-  case I:                                                                                                     \
-    return fp64 ? RankLayout<double, kNumGroups[I].TPR, kNumGroups[I].upper>::bytes(l1_words) + 1400         \
-                : RankLayout<float, kNumGroups[I].TPR, kNumGroups[I].upper>::bytes(l1_words) + 1400;
+#define SPG_G(I)                                                                                          \
+  case I:                                                                                                 \
+    return kStaticRankBytes +                                                                             \
+           (fp64 ? RankLayout<double, true, kNumGroups[I].TPR, kNumGroups[I].upper, kMetaPerThread,       \
+                              kNumKP>::bytes(l1_words)                                                    \
+                 : RankLayout<float, true, kNumGroups[I].TPR, kNumGroups[I].upper, kMetaPerThread,        \
+                              kNumKP>::bytes(l1_words));
     SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#undef SPG_G
+    default: return INT_MAX;
+  }
+}
+
+int rankcnt_smem_bytes(int group, int l1_words) {
+  switch (group) {
+#define SPG_G(I)                                                                                        \
+  case I:                                                                                               \
+    return kStaticRankBytes + RankLayout<int, false, kSymGroups[I].TPR, kSymGroups[I].upper,            \
+                                         kMetaPerThread,                                               \
+                                         sym_kp<kSymGroups[I].TPR, kSymGroups[I].upper>()>::bytes(l1_words);
+    SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return INT_MAX;
   }
@@ -284,6 +524,26 @@ int rankacc_smem_bytes(int group, bool fp64, int l1_words) {
 cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const NumArgs& a) {
   if (a.nrows <= 0) return cudaSuccess;
   return fp64 ? launch_rankacc_v<double>(s, group, a) : launch_rankacc_v<float>(s, group, a);
+}
+
+int rankbig_smem_bytes(bool fp64, int l1_words) {
+  return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_v<double>(l1_words) : rankbig_smem_bytes_v<float>(l1_words));
+}
+
+cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid) {
+  if (a.nrows <= 0 || grid <= 0) return cudaSuccess;
+  return fp64 ? launch_rankbig_v<double>(s, a, grid) : launch_rankbig_v<float>(s, a, grid);
+}
+
+cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a) {
+  if (a.nrows <= 0) return cudaSuccess;
+  switch (group) {
+#define SPG_G(I) \
+  case I: return launch_rankcnt_k<kSymGroups[I].TPR, kSymGroups[I].upper>(s, a);
+    SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#undef SPG_G
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 }  // namespace spg

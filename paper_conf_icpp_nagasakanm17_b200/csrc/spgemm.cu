@@ -623,6 +623,13 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.slab_T = slab_T;
   sa.nprod = static_cast<int64_t*>(h->nprod.p);
   sa.n = n;
+  sa.l1_words = (int)((n + 1023) / 1024 + 1);
+  sa.err_flags = &dacc->err_flags;
+  // rank-count kernels for the CTA-per-row groups (kernels_rankacc.cu; needs the column spans)
+  auto rank_cnt_on = [&](int g) {
+    return h->rank_acc && h->rlohi.p != nullptr && h->sym_min_group < 0 && g >= 5 && g <= 9 &&
+           rankcnt_smem_bytes(g, sa.l1_words) <= kSmemLimit;
+  };
   // range rows: pattern bitmap (symbolic -> numeric gather), rwcap words per row of the group
   const long long n_range = (long long)h->snap1.sym_rows[kSymRange];
   h->range_num = false;
@@ -650,7 +657,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   std::vector<long long> topo = {1, m, k, n, glob_grid, slab_T, h->vw_log2, sa.long_len, sa.flat, sa.fill_limit,
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
-                                 h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw};
+                                 h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
+                                 (long long)h->rank_acc};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -676,7 +684,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       SymArgs ga = sa;
       ga.rows = perm1 + off1.off[g];
       ga.nrows = rows;
-      CK(launch_symbolic_group(s, g, ga, h->num_sms));
+      if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
+      else CK(launch_symbolic_group(s, g, ga, h->num_sms));
       ++launches;
       if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
         SymArgs gb = sa;
@@ -840,15 +849,27 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const long long cwords = h->n / 32 + 2;
     const long long cstride = (2 * cwords * 4 + 255) & ~255LL;
     long long ccount[3] = {0, 0, 0}, ctotal = 0;
+    // rows above the CTA groups: rank-indexed accumulation with one CTA per row (level-2 bitmap
+    // and prefix in a per-CTA global slab of 8 B per output entry), else the DSMEM cluster tables
+    const bool big_rank = h->rank_acc && h->rlohi.p != nullptr && h->num_min_group < 0 &&
+                          rankbig_smem_bytes(fp64, l1w_rank) <= kSmemLimit;
+    long long bstride[3] = {0, 0, 0}, bgrid[3] = {0, 0, 0}, btotal = 0;
     for (int c = 0; c < 3; ++c) {
       const long long rows_c = (long long)h->snap2.num_rows[kNumCluster + c];
       if (rows_c == 0) continue;
+      if (big_rank) {
+        bstride[c] = (kNumGroups[kNumCluster + c].upper * 8 + 16 + 255) & ~255LL;
+        bgrid[c] = std::min<long long>(rows_c, h->num_sms);
+        btotal += bgrid[c] * bstride[c];
+        continue;
+      }
       int nc = 0;
       CK(launch_numeric_cluster(h->stream, fp64, 2 << c, na, &nc));
       ccount[c] = std::min<long long>(nc, rows_c);
       ctotal += ccount[c];
     }
     if (ctotal > 0) ALLOC(h->num_slab_c, (size_t)(ctotal * cstride));
+    if (btotal > 0) ALLOC(h->num_slab_c, (size_t)btotal);
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
     int glob_grid = 0;
     if (n_glob > 0) {
@@ -865,7 +886,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const int32_t* perm2 = static_cast<const int32_t*>(h->perm2.p);
     // phase 2 (per-group kernels on forked streams): captured once per key and replayed (e.g.
     // numeric re-runs with new values of the same structure, or repeated multiplies)
-    std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, h->vw_log2, na.long_len, na.flat,
+    std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, btotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
@@ -876,7 +897,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                          (long long)h->rbits.p, (long long)h->perm1.p};
     const bool ge = group_events(h);
     auto enqueue = [&]() -> spgemm_status_t {
-      if (ctotal > 0) CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
+      if (ctotal > 0 || btotal > 0) CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
       CK(fork(h));
       for (int g = 0; g < kNumNumGroups; ++g) {
         const long long rows = (long long)h->snap2.num_rows[g];
@@ -910,7 +931,17 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(cudaMalloc(&gc.prof, sizeof(unsigned long long) * 4 * rows));
             CK(cudaMemset(gc.prof, 0, sizeof(unsigned long long) * 4 * rows));
           }
-          CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
+          if (big_rank) {
+            long long boff = 0;
+            for (int q = 0; q < c; ++q) boff += bgrid[q] * bstride[q];
+            gc.slab = static_cast<unsigned char*>(h->num_slab_c.p) + boff;
+            gc.slab_stride = bstride[c];
+            gc.slab_T = (long long)kNumGroups[kNumCluster + c].upper;
+            gc.l1_words = l1w_rank;
+            CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c]));
+          } else {
+            CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
+          }
           if (gc.prof) {
             std::vector<unsigned long long> hp((size_t)(4 * rows));
             CK(cudaStreamSynchronize(st));

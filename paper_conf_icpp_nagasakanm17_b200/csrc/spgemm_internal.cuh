@@ -727,6 +727,8 @@ struct SymArgs {
   const int32_t* overflow2_rows;  // global kernel: rows that overflowed the cluster table
   const int* dev_count2;
   unsigned* rbits; long long rwcap;  // range rows: pattern bitmap, rwcap words per row of the group
+  int l1_words;            // rank-count kernels: level-1 words (>= n/1024 + 1)
+  int* err_flags;          // rank-count kernels: inconsistent-input flag (DevAcc::err_flags)
 };
 
 struct NumArgs {
@@ -778,6 +780,10 @@ cudaError_t launch_numeric_group(cudaStream_t s, int group, bool fp64, const Num
 cudaError_t launch_numeric_global(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
 cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const NumArgs& a);
 int rankacc_smem_bytes(int group, bool fp64, int l1_words);
+cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a);
+int rankcnt_smem_bytes(int group, int l1_words);
+cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
+int rankbig_smem_bytes(bool fp64, int l1_words);
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows);
 cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);

@@ -580,3 +580,28 @@ def test_rank_acc_duplicates_and_unsorted(spg):
         M.val[:] = M.val[o]
     got = check(spg, A, B, np.float64, what="dup/unsorted rank_acc")
     assert _rank_rows(got[3]) > 0
+
+
+def _big_rows(seed, m=240, k=1 << 17, n=1 << 21):
+    """Rows of C with 9K-60K entries over a ~2M-column span (numeric groups 10-12)."""
+    rng = np.random.default_rng(seed)
+    la = rng.integers(400, 2500, size=m)
+    rows = np.repeat(np.arange(m), la)
+    A = from_coo(m, k, rows, rng.integers(0, k, size=rows.size))
+    br = np.repeat(np.arange(k), 24)
+    B = from_coo(k, n, br, rng.integers(0, n, size=br.size))
+    return A, B
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_rank_acc_big_rows(spg, dtype):
+    A, B = _big_rows(31)
+    A, B = A.with_values("uniform", 1), B.with_values("uniform", 2)
+    got = check(spg, A, B, dtype, what="big rows rank")
+    assert sum(got[3]["num_rows"][10:13]) > 0, "no rows above the CTA groups"
+    check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
+
+
+def test_rank_acc_big_rows_int_exact(spg):
+    A, B = _big_rows(32)
+    check(spg, A.with_values("int", 3), B.with_values("int", 4), np.float32, exact=True, what="big rows int")
