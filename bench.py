@@ -137,14 +137,15 @@ def algorithmic_bytes(st: dict, phase: str, g: int, vbytes: int) -> int:
             + (4 + vbytes) * st["num_nnzc"][g] + 36 * st["num_rows"][g])
 
 
-def kernel_name(phase: str, g: int) -> str:
-    """Group -> kernel template as it appears in ncu / cuobjdump (spgemm_internal.cuh group ids)."""
+def kernel_name(phase: str, g: int, kind: int = 0) -> str:
+    """Group -> kernel template as it appears in ncu / cuobjdump (spgemm_internal.cuh group ids;
+    kind = spgemm_kernel_t the library reports for the group)."""
     if phase == "sym":
-        special = {11: "k_sym_global", 12: "k_sym_range"}
-        return f"{special.get(g, 'k_sym_smem<T,TPR,BS,OPT>')} (group {g})"
-    special = {10: "k_num_cluster<VT,2>", 11: "k_num_cluster<VT,4>", 12: "k_num_cluster<VT,8>",
-               13: "k_num_global<VT>", 14: "k_num_range<VT>"}
-    return f"{special.get(g, 'k_num_smem<VT,T,TPR,BS,UPPER>')} (group {g})"
+        k = {2: "k_sym_rankcnt<TPR,UPPER,KP,MC>", 3: "k_sym_range", 5: "k_sym_global"}.get(kind, "k_sym_smem<T,TPR,BS,OPT>")
+        return f"{k} (group {g})"
+    k = {2: "k_num_rankacc<VT,TPR,UPPER,KP,MC>", 3: "k_num_range<VT>", 4: "k_num_cluster<VT,CS>",
+         5: "k_num_global<VT>", 6: "k_num_rankbig<VT>"}.get(kind, "k_num_smem<VT,T,TPR,BS,UPPER>")
+    return f"{k} (group {g})"
 
 
 def load_peaks():
@@ -272,7 +273,8 @@ def run_ours(args):
     peak, peak_src = load_peaks()
     achieved = bytes_alg / (k_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": load_traffic(ph, g, args.dtype), "kernel": kernel_name(ph, g), "phase": ph, "group": g,
+                "traffic": load_traffic(ph, g, args.dtype),
+                "kernel": kernel_name(ph, g, st["sym_kernel" if ph == "sym" else "num_kernel"][g]), "phase": ph, "group": g,
                 "launch_ms": k_ms, "share_of_step": k_ms / (tot_ms / args.steps),
                 "algorithmic_bytes_per_launch": bytes_alg, "peak_source": peak_src}
 

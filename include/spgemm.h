@@ -187,7 +187,20 @@ typedef struct {
     int64_t workspace_bytes, workspace_peak_bytes;
     int64_t sym_overflow2_rows;         /* rows that overflowed the cluster table (global memory) */
     int64_t graph_replays;              /* captured segments replayed during the last call pair */
+    int32_t sym_kernel[SPGEMM_MAX_GROUPS];  /* kernel family that ran each group of the last call: */
+    int32_t num_kernel[SPGEMM_MAX_GROUPS];  /* spgemm_kernel_t below (0: group empty / not run)    */
 } spgemm_stats_t;
+
+/* Kernel families reported per group in spgemm_stats_t. */
+typedef enum {
+    SPGEMM_KERNEL_NONE = 0,
+    SPGEMM_KERNEL_HASH = 1,     /* paper hash table in shared memory (Alg. 5, Table I groups)    */
+    SPGEMM_KERNEL_RANK = 2,     /* rank-indexed table, one CTA per row (kernels_rankacc.cu)      */
+    SPGEMM_KERNEL_RANGE = 3,    /* range rows: offset table, warp per row (kernels_range.cu)     */
+    SPGEMM_KERNEL_CLUSTER = 4,  /* distributed shared-memory hash table (kernels_cluster.cu)     */
+    SPGEMM_KERNEL_GLOBAL = 5,   /* global-memory hash table                  */
+    SPGEMM_KERNEL_RANK_BIG = 6  /* rank-indexed, level 2 in global memory, values reduced into C */
+} spgemm_kernel_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);
 

@@ -28,6 +28,9 @@ OPTIONS = {
     "range_min_nprod": 15, "bitmap_rank": 16, "rank_acc": 17,
 }
 
+# spgemm_kernel_t (include/spgemm.h): kernel family that ran each group
+KERNELS = {0: "none", 1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big"}
+
 # Group ids of the range-row kernels (spgemm_internal.cuh kSymRange / kNumRange).
 SYM_RANGE_GROUP = 12
 NUM_RANGE_GROUP = 14
@@ -65,6 +68,7 @@ class Stats(ctypes.Structure):
         ("kernel_launches_symbolic", c_int64), ("kernel_launches_numeric", c_int64),
         ("workspace_bytes", c_int64), ("workspace_peak_bytes", c_int64),
         ("sym_overflow2_rows", c_int64), ("graph_replays", c_int64),
+        ("sym_kernel", c_int32 * G), ("num_kernel", c_int32 * G),
     ]
 
     def to_dict(self) -> dict:

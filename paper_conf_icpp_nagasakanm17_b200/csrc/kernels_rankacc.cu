@@ -124,8 +124,21 @@ struct RankLayout {
   static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1w * 2); }
 };
 
-constexpr int kMetaPerThread = 2;
-__host__ __device__ constexpr int rankbig_l1pad_h(int l1w) { return (l1w + 3) & ~3; }  // MC: A non-zeros of a row held as metadata per thread
+// Per-group launch shape of the rank kernels (independent of the hash groups' Table-I shapes):
+// TPR threads (one row per CTA), KP products per thread held in registers (fast path: n_prod_i <=
+// KP*TPR), MC A non-zeros of metadata per thread (fast path: nnz(A_i) <= MC*TPR).  Numeric groups
+// are keyed by nnz_i (graph rows: n_prod_i ~ nnz_i, so KP*TPR >= the bound), symbolic groups by
+// n_prod_i (KP*TPR = the bound).
+struct RankCfg {
+  int TPR, KP, MC;
+};
+constexpr RankCfg kRankNum[] = {{0, 0, 0},   {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},
+                                {128, 8, 2}, {256, 8, 2},  {512, 8, 2},  {512, 9, 2},  {1024, 9, 2}};
+// symbolic groups 3-4 stay on the paper hash (faster there: measured R-MAT s20 0.28/0.66 ms vs
+// 0.53/0.69 ms); MC 4 measured slower than 2 for groups 5-8
+constexpr RankCfg kRankSym[] = {{0, 0, 0},    {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},
+                                {64, 16, 2},  {128, 16, 2}, {256, 16, 2}, {512, 16, 2}, {1024, 16, 2}};
+__host__ __device__ constexpr int rankbig_l1pad_h(int l1w) { return (l1w + 3) & ~3; }
 
 // Adapters so rank_row reads both argument structs the same way.
 struct NumView : NumArgs {
@@ -138,10 +151,9 @@ struct SymView : SymArgs {
 };
 
 // One row, symbolic (NUM = false: writes nnz_i to c_cnt[row]) or numeric (writes the row of C).
-template <typename VT, bool NUM, int TPR, long long UPPER, int KP, typename Args>
+template <typename VT, bool NUM, int TPR, long long UPPER, int KP, int MC, typename Args>
 __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* smem_raw, int (*ws32)[32],
                                          long long* ws64) {
-  constexpr int MC = kMetaPerThread;
   using L = RankLayout<VT, NUM, TPR, UPPER, MC, KP>;
   constexpr int ME = L::ME;
   VT* vals = reinterpret_cast<VT*>(smem_raw + L::kVals);
@@ -200,9 +212,12 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
 
   int key[KP];
   VT val[KP];
+  // set-if-clear: rows that compress (duplicate columns) would otherwise serialise on the same
+  // words; a stale read only costs a redundant atomic
   auto set_l1 = [&](int k) {
     const unsigned d = (unsigned)(k - lo);
-    atomicOr(l1 + (d >> 10), 1u << ((d >> 5) & 31));
+    const unsigned bit = 1u << ((d >> 5) & 31);
+    if (!(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
   };
   auto blk_of = [&](unsigned d) {
     const unsigned w = d >> 10, bit = (d >> 5) & 31;
@@ -210,7 +225,9 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   };
   auto set_fine = [&](int k) {
     const unsigned d = (unsigned)(k - lo);
-    atomicOr(fine + blk_of(d), 1u << (d & 31));
+    const int b = blk_of(d);
+    const unsigned bit = 1u << (d & 31);
+    if (!(fine[b] & bit)) atomicOr(fine + b, bit);
   };
   auto accumulate = [&](int k, VT v) {
     const unsigned d = (unsigned)(k - lo);
@@ -307,25 +324,21 @@ constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 
 template <int TPR, int VB>
 constexpr int rank_min_blocks() { return TPR >= 1024 ? 1 : (VB > 4 ? 1024 : 1536) / TPR; }
 
-template <typename VT, int TPR, long long UPPER, int KP>
+template <typename VT, int TPR, long long UPPER, int KP, int MC>
 __global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT)>()) void k_num_rankacc(NumArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];
-  rank_row<VT, true, TPR, UPPER, KP>(static_cast<const NumView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
+  rank_row<VT, true, TPR, UPPER, KP, MC>(static_cast<const NumView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
 }
 
-template <int TPR, long long UPPER, int KP>
+template <int TPR, long long UPPER, int KP, int MC>
 __global__ __launch_bounds__(TPR, rank_min_blocks<TPR, 4>()) void k_sym_rankcnt(SymArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];
-  rank_row<int, false, TPR, UPPER, KP>(static_cast<const SymView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
+  rank_row<int, false, TPR, UPPER, KP, MC>(static_cast<const SymView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
 }
-
-constexpr int kNumKP = 8;
-template <int TPR, long long UPPER>
-constexpr int sym_kp() { return (int)(UPPER / TPR) > 16 ? 16 : (int)(UPPER / TPR); }
 
 template <typename K>
 cudaError_t prepare(K kernel, int smem, int& configured) {
@@ -340,26 +353,29 @@ cudaError_t prepare(K kernel, int smem, int& configured) {
   return cudaSuccess;
 }
 
-template <typename VT, int TPR, long long UPPER>
+template <typename VT, int G>
 cudaError_t launch_rankacc_k(cudaStream_t s, const NumArgs& a) {
-  using L = RankLayout<VT, true, TPR, UPPER, kMetaPerThread, kNumKP>;
+  constexpr RankCfg c = kRankNum[G];
+  constexpr long long UPPER = kNumGroups[G].upper;
+  using L = RankLayout<VT, true, c.TPR, UPPER, c.MC, c.KP>;
   const int smem = L::bytes(a.l1_words);
   static int configured = 0;
-  cudaError_t e = prepare(k_num_rankacc<VT, TPR, UPPER, kNumKP>, smem, configured);
+  cudaError_t e = prepare(k_num_rankacc<VT, c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
-  k_num_rankacc<VT, TPR, UPPER, kNumKP><<<(unsigned)a.nrows, TPR, smem, s>>>(a);
+  k_num_rankacc<VT, c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
   return cudaGetLastError();
 }
 
-template <int TPR, long long UPPER>
+template <int G>
 cudaError_t launch_rankcnt_k(cudaStream_t s, const SymArgs& a) {
-  constexpr int KP = sym_kp<TPR, UPPER>();
-  using L = RankLayout<int, false, TPR, UPPER, kMetaPerThread, KP>;
+  constexpr RankCfg c = kRankSym[G];
+  constexpr long long UPPER = kSymGroups[G].upper;
+  using L = RankLayout<int, false, c.TPR, UPPER, c.MC, c.KP>;
   const int smem = L::bytes(a.l1_words);
   static int configured = 0;
-  cudaError_t e = prepare(k_sym_rankcnt<TPR, UPPER, KP>, smem, configured);
+  cudaError_t e = prepare(k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
-  k_sym_rankcnt<TPR, UPPER, KP><<<(unsigned)a.nrows, TPR, smem, s>>>(a);
+  k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -367,8 +383,8 @@ template <typename VT>
 cudaError_t launch_rankacc_v(cudaStream_t s, int group, const NumArgs& a) {
   switch (group) {
 #define SPG_G(I) \
-  case I: return launch_rankacc_k<VT, kNumGroups[I].TPR, kNumGroups[I].upper>(s, a);
-    SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+  case I: return launch_rankacc_k<VT, I>(s, a);
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return cudaErrorInvalidValue;
   }
@@ -448,7 +464,8 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
     __syncthreads();
     walk([&](int k, VT) {
       const unsigned d = (unsigned)(k - lo);
-      atomicOr(l1 + (d >> 10), 1u << ((d >> 5) & 31));
+      const unsigned bit = 1u << ((d >> 5) & 31);
+      if (!(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
     });
     __syncthreads();
     const int nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
@@ -495,14 +512,14 @@ constexpr int kStaticRankBytes = 2 * 32 * 4 + 33 * 8 + 1024;  // static shared +
 
 int rankacc_smem_bytes(int group, bool fp64, int l1_words) {
   switch (group) {
-#define SPG_G(I)                                                                                          \
-  case I:                                                                                                 \
-    return kStaticRankBytes +                                                                             \
-           (fp64 ? RankLayout<double, true, kNumGroups[I].TPR, kNumGroups[I].upper, kMetaPerThread,       \
-                              kNumKP>::bytes(l1_words)                                                    \
-                 : RankLayout<float, true, kNumGroups[I].TPR, kNumGroups[I].upper, kMetaPerThread,        \
-                              kNumKP>::bytes(l1_words));
-    SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#define SPG_G(I)                                                                                     \
+  case I:                                                                                            \
+    return kStaticRankBytes +                                                                        \
+           (fp64 ? RankLayout<double, true, kRankNum[I].TPR, kNumGroups[I].upper, kRankNum[I].MC,    \
+                              kRankNum[I].KP>::bytes(l1_words)                                       \
+                 : RankLayout<float, true, kRankNum[I].TPR, kNumGroups[I].upper, kRankNum[I].MC,     \
+                              kRankNum[I].KP>::bytes(l1_words));
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return INT_MAX;
   }
@@ -510,12 +527,11 @@ int rankacc_smem_bytes(int group, bool fp64, int l1_words) {
 
 int rankcnt_smem_bytes(int group, int l1_words) {
   switch (group) {
-#define SPG_G(I)                                                                                        \
-  case I:                                                                                               \
-    return kStaticRankBytes + RankLayout<int, false, kSymGroups[I].TPR, kSymGroups[I].upper,            \
-                                         kMetaPerThread,                                               \
-                                         sym_kp<kSymGroups[I].TPR, kSymGroups[I].upper>()>::bytes(l1_words);
-    SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#define SPG_G(I)                                                                                  \
+  case I:                                                                                         \
+    return kStaticRankBytes + RankLayout<int, false, kRankSym[I].TPR, kSymGroups[I].upper,        \
+                                         kRankSym[I].MC, kRankSym[I].KP>::bytes(l1_words);
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return INT_MAX;
   }
@@ -539,8 +555,8 @@ cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a)
   if (a.nrows <= 0) return cudaSuccess;
   switch (group) {
 #define SPG_G(I) \
-  case I: return launch_rankcnt_k<kSymGroups[I].TPR, kSymGroups[I].upper>(s, a);
-    SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+  case I: return launch_rankcnt_k<I>(s, a);
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
 #undef SPG_G
     default: return cudaErrorInvalidValue;
   }

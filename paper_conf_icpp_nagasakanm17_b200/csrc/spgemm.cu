@@ -38,6 +38,7 @@ struct GraphCache {
   std::vector<long long> topo;   // topology key: launch structure only (grids, groups, options)
   int launches = 0;              // kernels in the captured segment
   bool timed[16] = {};           // groups with timing events in the segment
+  int kind[16] = {};             // spgemm_kernel_t of every group in the segment
 };
 
 struct DeviceGuard {
@@ -74,6 +75,7 @@ struct spgemm_ctx {
   cudaEvent_t ev[8]{};
   cudaEvent_t gstart[2][kMaxGroups]{}, gstop[2][kMaxGroups]{};
   bool gtimed[2][kMaxGroups]{};
+  int gkind[2][kMaxGroups]{};    // spgemm_kernel_t per group of the last call (stats)
   bool gtimed_phases = false;  // ev[1], ev[2] recorded (per-group events on)
   // options
   int sym_min_group = -1, num_min_group = -1, fill_limit = 0, use_streams = 1, validate = 0, lanes = 0;
@@ -534,6 +536,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   h->a_rpt = a_rpt; h->a_col = a_col; h->b_rpt = b_rpt; h->b_col = b_col; h->c_rpt = c_rpt;
   memset(&h->stats, 0, sizeof h->stats);
   memset(h->gtimed, 0, sizeof h->gtimed);
+  memset(h->gkind, 0, sizeof h->gkind);
   h->ws_peak = h->ws_cur;
   h->stats.m = m; h->stats.k = k; h->stats.n = n;
   h->stats.n_sym_groups = kNumSymGroups;
@@ -686,6 +689,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       ga.nrows = rows;
       if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
       else CK(launch_symbolic_group(s, g, ga, h->num_sms));
+      h->gkind[0][g] = rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
       ++launches;
       if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
         SymArgs gb = sa;
@@ -707,6 +711,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
         }
         CK(launch_symbolic_global(s, gb, glob_grid));
         ++launches;
+        if (glob_grid > 0) h->gkind[0][kSymGlobal] = SPGEMM_KERNEL_GLOBAL;
       }
       if (ge) CK(cudaEventRecord(h->gstop[0][g], s));
       h->gtimed[0][g] = ge;
@@ -729,6 +734,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       }
       if (ge) CK(cudaEventRecord(h->gstop[0][kSymRange], s));
       h->gtimed[0][kSymRange] = ge;
+      h->gkind[0][kSymRange] = SPGEMM_KERNEL_RANGE;
     }
     if (n_opt == 0 && n_glob > 0) {  // forced global group only
       cudaStream_t s = group_stream(h, kSymGlobal);
@@ -741,6 +747,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       ++launches;
       if (ge) CK(cudaEventRecord(h->gstop[0][kSymGlobal], s));
       h->gtimed[0][kSymGlobal] = ge;
+      h->gkind[0][kSymGlobal] = SPGEMM_KERNEL_GLOBAL;
     }
     CK(join(h));
     if (ge) CK(cudaEventRecord(h->ev[2], h->stream));
@@ -763,9 +770,11 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
     if (seg_launches < 0) {  // replayed without enqueueing
       seg_launches = h->gsym.launches;
       memcpy(h->gtimed[0], h->gsym.timed, sizeof h->gsym.timed);
+      memcpy(h->gkind[0], h->gsym.kind, sizeof h->gsym.kind);
     } else {
       h->gsym.launches = seg_launches;
       memcpy(h->gsym.timed, h->gtimed[0], sizeof h->gsym.timed);
+      memcpy(h->gsym.kind, h->gkind[0], sizeof h->gsym.kind);
     }
   }
   launches += seg_launches;
@@ -817,6 +826,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
   CK(enter(h));
   h->stats.kernel_launches_numeric = 0;
   memset(h->gtimed[1], 0, sizeof h->gtimed[1]);
+  memset(h->gkind[1], 0, sizeof h->gkind[1]);
   h->numeric_done = true;
   if (h->timing) CK(cudaEventRecord(h->ev[4], h->stream));
   if (h->m > 0 && h->nnzc > 0) {
@@ -841,8 +851,13 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // rank-indexed accumulation for the CTA-per-row groups (needs the column spans; the forced
     // paths keep the paper hash)
     const int l1w_rank = (int)((h->n + 1023) / 1024 + 1);
+    // The CTA-group rank kernels hold <= KP*TPR (>= 2x the group's nnz bound) products per row in
+    // registers; rows beyond that re-walk their products three times, which loses to the paper
+    // hash when rows compress well (QCD-like: n_prod/nnz = 7.2).  Decided per call from the
+    // global compression n_prod / nnz(C) (known at sync 2).
+    const bool low_compression = (double)h->snap1.total_nprod <= 2.5 * (double)h->nnzc;
     auto rank_acc_on = [&](int g) {
-      return h->rank_acc && h->rlohi.p != nullptr && h->num_min_group < 0 && g >= 4 && g <= 9 &&
+      return h->rank_acc && low_compression && h->rlohi.p != nullptr && h->num_min_group < 0 && g >= 3 && g <= 9 &&
              rankacc_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit;
     };
     // cluster groups (clusters of 2/4/8 CTAs): bitmap + prefix scratch per resident cluster
@@ -888,7 +903,8 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // numeric re-runs with new values of the same structure, or repeated multiplies)
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, btotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
-                                   h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc};
+                                   h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc,
+                                   (long long)low_compression};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
@@ -908,6 +924,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
         ga.rows = perm2 + off2.off[g];
         ga.nrows = rows;
         if (g == kNumGlobal) {
+          h->gkind[1][g] = SPGEMM_KERNEL_GLOBAL;
           CK(launch_numeric_global(st, fp64, ga, glob_grid));
         } else if (g == kNumRange) {
           // the symbolic range rows in their phase-1 order (the bitmap's row index)
@@ -916,6 +933,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
           ra.nrows = (long long)h->snap1.sym_rows[kSymRange];
           ra.rbits = static_cast<const unsigned*>(h->rbits.p);
           ra.rwcap = range_wcap(h->snap1.range_rmax);
+          h->gkind[1][g] = SPGEMM_KERNEL_RANGE;
           CK(launch_numeric_range(st, fp64, ra, h->snap1.range_rmax, h->num_sms));
         } else if (g >= kNumCluster && g < kNumCluster + 3) {
           const int c = g - kNumCluster;
@@ -939,8 +957,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             gc.slab_T = (long long)kNumGroups[kNumCluster + c].upper;
             gc.l1_words = l1w_rank;
             CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c]));
+            h->gkind[1][g] = SPGEMM_KERNEL_RANK_BIG;
           } else {
             CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
+            h->gkind[1][g] = SPGEMM_KERNEL_CLUSTER;
           }
           if (gc.prof) {
             std::vector<unsigned long long> hp((size_t)(4 * rows));
@@ -963,8 +983,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             NumArgs ra = ga;
             ra.l1_words = l1w_rank;
             CK(launch_numeric_rankacc(st, g, fp64, ra));
+            h->gkind[1][g] = SPGEMM_KERNEL_RANK;
           } else {
             CK(launch_numeric_group(st, g, fp64, ga));
+            h->gkind[1][g] = SPGEMM_KERNEL_HASH;
           }
           if (ga.prof) {
             std::vector<unsigned long long> hp((size_t)(4 * rows));
@@ -991,9 +1013,11 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     if (h->stats.kernel_launches_numeric == before_launches) {  // replayed without enqueueing
       h->stats.kernel_launches_numeric += h->gnum.launches;
       memcpy(h->gtimed[1], h->gnum.timed, sizeof h->gnum.timed);
+      memcpy(h->gkind[1], h->gnum.kind, sizeof h->gnum.kind);
     } else {
       h->gnum.launches = (int)(h->stats.kernel_launches_numeric - before_launches);
       memcpy(h->gnum.timed, h->gtimed[1], sizeof h->gnum.timed);
+      memcpy(h->gnum.kind, h->gkind[1], sizeof h->gnum.kind);
     }
   }
   if (h->timing) CK(cudaEventRecord(h->ev[5], h->stream));
@@ -1006,6 +1030,10 @@ spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t* out) {
   DeviceGuard dg(h->device);
   CK(enter(h));
   spgemm_stats_t st = h->stats;
+  for (int g = 0; g < kMaxGroups; ++g) {
+    st.sym_kernel[g] = h->gkind[0][g];
+    st.num_kernel[g] = h->numeric_done ? h->gkind[1][g] : 0;
+  }
   if (h->state == 1 && h->m > 0 && h->timing) {
     auto el = [&](cudaEvent_t a, cudaEvent_t b) -> float {
       float ms = 0.f;

@@ -43,6 +43,16 @@ def group_of(kname: str):
     if m:
         T, TPR, BS, up = int(m.group(2)), int(m.group(3)), int(m.group(4)), int(m.group(5))
         return "num", NUM.get((T, TPR, BS, up))
+    m = re.search(r"k_num_rankacc<\w+, (?:\(int\))?(\d+), (?:\(long long\))?(\d+)", kname)
+    if m:
+        up = int(m.group(2))
+        return "num", next((g for (t, tpr, bs, u), g in NUM.items() if u == up), None)
+    m = re.search(r"k_sym_rankcnt<(?:\(int\))?(\d+), (?:\(long long\))?(\d+)", kname)
+    if m:
+        up = int(m.group(2))
+        return "sym", next((g for (t, tpr, bs, u), g in SYM.items() if u == up), None)
+    if "k_num_rankbig" in kname:
+        return "num", 10
     if re.search(r"k_sym_range(_bits)?\b", kname):
         return "sym", 12  # kSymRange
     if "k_num_range" in kname:

@@ -551,9 +551,20 @@ def test_rank_acc_vs_paper_hash(spg, name, dtype):
     A = _mixed_small() if name == "webbase_small" else (
         synth.rmat(14).with_values("uniform", 9) if name == "rmat14" else synth.config(name))
     got = check(spg, A, A, dtype, what=f"{name} rank_acc")
+    st = got[3]
     if name != "mixed:circuit":
-        assert _rank_rows(got[3]) > 0, "no rows in the rank-accumulate groups"
-    check(spg, A, A, dtype, opts={"rank_acc": 0}, what=f"{name} paper hash")
+        assert _rank_rows(st) > 0, "no rows in the rank-accumulate groups"
+    # kernel family per group (spgemm_kernel_t): rank for low-compression inputs, the paper hash
+    # for the QCD-like rows (n_prod/nnz = 7.2), rank counts for symbolic groups 5-9 either way
+    want = 1 if name == "mixed:qcd" else 2
+    for g in range(3, 10):
+        if st["num_rows"][g]:
+            assert st["num_kernel"][g] == want, (g, st["num_kernel"])
+    for g in range(5, 10):
+        if st["sym_rows"][g]:
+            assert st["sym_kernel"][g] == 2, (g, st["sym_kernel"])
+    got = check(spg, A, A, dtype, opts={"rank_acc": 0}, what=f"{name} paper hash")
+    assert all(k in (0, 1, 3, 4, 5) for k in got[3]["num_kernel"][:13]), got[3]["num_kernel"]
 
 
 @pytest.mark.parametrize("name", ["rmat14", "mixed:qcd"])
