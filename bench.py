@@ -56,6 +56,8 @@ def parse():
     p.add_argument("--cpu-runs", type=int, default=5)
     p.add_argument("--lanes", type=int, default=0, help="lanes per B row (0 = library auto)")
     p.add_argument("--streams", type=int, default=1)
+    p.add_argument("--opt", action="append", default=[],
+                   help="library option name=value (ablations, e.g. rank_acc=0; see _lib.OPTIONS)")
     return p.parse_args()
 
 
@@ -74,7 +76,8 @@ def config_dict(args, A, world):
     return {"workload": f"{args.config}-like A^2" if args.config != "poisson64" else "poisson64 A^2",
             "matrix": A.name, "rows": A.m, "nnz_a": A.nnz, "dtype": args.dtype,
             "per_rank": "row block p of diag(A_0..A_{N-1})^2 (weak scaling)" if world > 1 else "single GPU",
-            "l2": "flushed (512 MiB write) before every timed step", "inputs": "device-resident (value)"}
+            "l2": "flushed (512 MiB write) before every timed step", "inputs": "device-resident (value)",
+            **({"options": dict(o.split("=") for o in args.opt)} if getattr(args, "opt", None) else {})}
 
 
 # ----------------------------------------------------------------------------- clocks
@@ -211,6 +214,9 @@ def run_ours(args):
     # per-group kernel events over the timed region (timing=2 runs the group kernels eagerly; the
     # CUDA-graph replay mode is timed separately below and reported as `graph_replay`)
     h.set_option("lanes", args.lanes).set_option("streams", args.streams).set_option("timing", 2)
+    for o in args.opt:
+        k, v = o.split("=")
+        h.set_option(k, int(v))
     dA = P.CsrMatrix.from_host(A, dev, tdt)
     stream = h.stream
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
