@@ -132,10 +132,12 @@ struct RankLayout {
 struct RankCfg {
   int TPR, KP, MC;
 };
-// numeric: KP*TPR = the nnz bound for groups 5-8 (graph rows' n_prod_i is within ~1 % of nnz_i;
+// numeric: KP*TPR = the nnz bound for groups 6-8 (graph rows' n_prod_i is within ~1 % of nnz_i;
 // the few rows above it take the re-walk path) — half the warps per row of KP*TPR = 2x the bound
-constexpr RankCfg kRankNum[] = {{0, 0, 0},  {0, 0, 0},   {0, 0, 0},   {64, 4, 2},  {64, 8, 2},
-                                {64, 8, 2}, {128, 8, 2}, {256, 8, 2}, {512, 8, 2}, {1024, 9, 2}};
+// (R-MAT s20: groups 6-8 1.86/2.21/1.90 -> 1.73/1.69/1.82 ms); group 5 keeps 128 threads (64:
+// the span-sized level-1 bitmap per CTA limits residency, 1.21 -> 1.38 ms)
+constexpr RankCfg kRankNum[] = {{0, 0, 0},   {0, 0, 0},   {0, 0, 0},   {64, 4, 2},  {64, 8, 2},
+                                {128, 8, 2}, {128, 8, 2}, {256, 8, 2}, {512, 8, 2}, {1024, 9, 2}};
 // symbolic groups 3-4 stay on the paper hash (faster there: measured R-MAT s20 0.28/0.66 ms vs
 // 0.53/0.69 ms); MC 4 measured slower than 2 for groups 5-8
 constexpr RankCfg kRankSym[] = {{0, 0, 0},    {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},

@@ -87,7 +87,8 @@ struct spgemm_ctx {
   int timing = 1;
   int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
   long long range_min_np = kRangeMinNprodDefault;
-  int rank_acc = 1;      // CTA-per-row numeric groups: rank-indexed accumulation (kernels_rankacc.cu)
+  int rank_acc = 1;
+  bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)      // CTA-per-row numeric groups: rank-indexed accumulation (kernels_rankacc.cu)
   int bitmap_rank = 1;   // CTA-per-row numeric groups: two-level bitmap rank (else bucket sort)
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -297,17 +298,24 @@ cudaError_t leave(spgemm_handle_t h) {
   return e == cudaSuccess ? cudaStreamWaitEvent(h->ustream, h->ev_leave, 0) : e;
 }
 
-cudaStream_t group_stream(spgemm_handle_t h, int g) { return h->use_streams ? h->gs[g % kNumStreams] : h->stream; }
+// Per-group streams only when the phase has >= 2 non-empty groups (one group: the fork/join
+// events cost ~3 % of the cant step for nothing).
+bool phase_concurrent(spgemm_handle_t h, const unsigned long long* rows, int ngroups) {
+  int ne = 0;
+  for (int g = 0; g < ngroups; ++g) ne += rows[g] > 0;
+  return h->use_streams && ne >= 2;
+}
+cudaStream_t group_stream(spgemm_handle_t h, int g) { return h->phase_streams ? h->gs[g % kNumStreams] : h->stream; }
 
 cudaError_t fork(spgemm_handle_t h) {
-  if (!h->use_streams) return cudaSuccess;
+  if (!h->phase_streams) return cudaSuccess;
   cudaError_t e = cudaEventRecord(h->fork_ev, h->stream);
   for (int i = 0; i < kNumStreams && e == cudaSuccess; ++i) e = cudaStreamWaitEvent(h->gs[i], h->fork_ev, 0);
   return e;
 }
 
 cudaError_t join(spgemm_handle_t h) {
-  if (!h->use_streams) return cudaSuccess;
+  if (!h->phase_streams) return cudaSuccess;
   cudaError_t e = cudaSuccess;
   for (int i = 0; i < kNumStreams && e == cudaSuccess; ++i) {
     e = cudaEventRecord(h->join_ev[i], h->gs[i]);
@@ -678,6 +686,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                             static_cast<int32_t*>(h->perm1.p)));
     ++launches;
     if (ge) CK(cudaEventRecord(h->ev[1], h->stream));
+    h->phase_streams = phase_concurrent(h, h->snap1.sym_rows, kNumSymGroups);
     CK(fork(h));
     for (int g = 0; g <= kSymOptimistic; ++g) {
       const long long rows = (long long)h->snap1.sym_rows[g];
@@ -914,6 +923,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const bool ge = group_events(h);
     auto enqueue = [&]() -> spgemm_status_t {
       if (ctotal > 0 || btotal > 0) CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
+      h->phase_streams = phase_concurrent(h, h->snap2.num_rows, kNumNumGroups);
       CK(fork(h));
       for (int g = 0; g < kNumNumGroups; ++g) {
         const long long rows = (long long)h->snap2.num_rows[g];
