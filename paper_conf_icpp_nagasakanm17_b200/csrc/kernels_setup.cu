@@ -53,17 +53,41 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, cons
   const int G = 1 << glog, lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int rpc = kSetupThreads >> glog;
   bool bad = false;
-  for (long long blk = (long long)blockIdx.x * rpc; blk < k; blk += (long long)gridDim.x * rpc) {
-    const long long row = blk + (threadIdx.x >> glog);
+  // One lane per row (mean row length < 8, power-law shapes): rows interleaved over CTAs (row =
+  // base + slot * gridDim.x + blockIdx.x) — long rows cluster in index ranges, and contiguous
+  // slices hand one warp many of them in series (webbase: 152 -> 119 us; with G > 1 the
+  // contiguous slices' coalesced rpt loads win: cant 25 -> 31 us, R-MAT 241 -> 267 us interleaved)
+  const long long T = (long long)gridDim.x * rpc;
+  const bool ilv = G == 1;
+  for (long long base = 0; base < k; base += T) {
+    const long long row = base + (ilv ? (long long)(threadIdx.x >> glog) * gridDim.x + blockIdx.x
+                                      : (long long)blockIdx.x * rpc + (threadIdx.x >> glog));
     long long b0 = 0, b1 = 0;
     if (row < k) { b0 = __ldg(b_rpt + row); b1 = __ldg(b_rpt + row + 1); }
     const bool is_long = b1 - b0 > (long long)kLongPerLane * G;
     int mn = INT_MAX, mx = -1;
     if (!is_long) {
-      for (long long j = b0 + gl; j < b1; j += G) {
-        const int c = __ldg(b_col + j);
-        mn = min(mn, c); mx = max(mx, c);
-        if (j > b0) bad |= c <= __ldg(b_col + j - 1);
+      // 4 entries per lane per step, all loads issued first; the predecessor of entry j (for the
+      // strictly-increasing check) is the previous lane's entry (shuffle), or for lane 0 the last
+      // lane's entry of the previous slot
+      const unsigned gm = G >= 32 ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+      int carry = INT_MIN;  // entry j-1 of lane 0's first slot (none before the row start)
+      for (long long j = b0 + gl; j - gl < b1; j += 4 * G) {  // G-uniform trip count
+        int c[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) c[u] = j + u * G < b1 ? __ldg(b_col + j + u * G) : INT_MAX;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const bool in = j + u * G < b1;
+          int prev = __shfl_up_sync(gm, c[u], 1, G);
+          const int last = __shfl_sync(gm, c[u], G - 1, G);
+          if (gl == 0) prev = carry;
+          carry = last;
+          if (in) {
+            mn = min(mn, c[u]); mx = max(mx, c[u]);
+            bad |= prev != INT_MIN && c[u] <= prev;
+          }
+        }
       }
     }
     for (int o = G >> 1; o > 0; o >>= 1) {
@@ -77,10 +101,20 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, cons
       const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
       int pmn = INT_MAX, pmx = -1;
       bool pbad = false;
-      for (long long j = s0 + lane; j < s1; j += 32) {
-        const int c = __ldg(b_col + j);
-        pmn = min(pmn, c); pmx = max(pmx, c);
-        if (j > s0) pbad |= c <= __ldg(b_col + j - 1);
+      for (long long j = s0 + lane; j < s1; j += 8 * 32) {  // 8 loads (+8 predecessors) in flight
+        int c[8], pv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const long long q = j + 32 * u;
+          c[u] = q < s1 ? __ldg(b_col + q) : 0;
+          pv[u] = q < s1 && q > s0 ? __ldg(b_col + q - 1) : INT_MIN;
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+          if (j + 32 * u < s1) {
+            pmn = min(pmn, c[u]); pmx = max(pmx, c[u]);
+            pbad |= pv[u] != INT_MIN && c[u] <= pv[u];
+          }
       }
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) {
@@ -115,8 +149,11 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
   const bool b_ok = bd.range_group >= 0 && __ldg(b_rpt + bd.range_k) < (1LL << 31);
   unsigned long long tot = 0, mxnp = 0;
   int span_max = 0;
-  for (long long blk = (long long)blockIdx.x * rpc; blk < m; blk += (long long)gridDim.x * rpc) {
-    const long long row = blk + (threadIdx.x >> glog);
+  const long long T = (long long)gridDim.x * rpc;  // rows interleaved over CTAs when G = 1 (see k_brow_minmax)
+  const bool ilv = G == 1;
+  for (long long base = 0; base < m; base += T) {
+    const long long row = base + (ilv ? (long long)(threadIdx.x >> glog) * gridDim.x + blockIdx.x
+                                      : (long long)blockIdx.x * rpc + (threadIdx.x >> glog));
     long long a0 = 0, a1 = 0;
     if (row < m) { a0 = __ldg(a_rpt + row); a1 = __ldg(a_rpt + row + 1); }
     const bool is_long = a1 - a0 > (long long)kLongPerLane * G;
@@ -148,10 +185,16 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
       const long long s0 = __shfl_sync(0xffffffffu, a0, src), s1 = __shfl_sync(0xffffffffu, a1, src);
       long long part = 0;
       int plo = INT_MAX, phi = -1;
-      for (long long j = s0 + lane; j < s1; j += 32) {
-        const int kk = __ldg(a_col + j);
-        part += __ldg(b_rpt + kk + 1) - __ldg(b_rpt + kk);
-        if (bmm) { const int2 r = __ldg(bmm + kk); plo = min(plo, r.x); phi = max(phi, r.y); }
+      for (long long j = s0 + lane; j < s1; j += 8 * 32) {  // 8 entries per lane in flight
+        int kk[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) kk[u] = j + 32 * u < s1 ? __ldg(a_col + j + 32 * u) : -1;
+#pragma unroll
+        for (int u = 0; u < 8; ++u)
+          if (kk[u] >= 0) {
+            part += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+            if (bmm) { const int2 r = __ldg(bmm + kk[u]); plo = min(plo, r.x); phi = max(phi, r.y); }
+          }
       }
       part = (long long)warp_sum_u64((unsigned long long)part);
 #pragma unroll
