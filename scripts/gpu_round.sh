@@ -4,7 +4,7 @@
 # capture of the hot group kernels of one bench step.
 #   bash scripts/gpu_round.sh TAG [KREGEX]
 TAG=${1:-r01}
-KRE=${2:-'k_(num|sym)_(smem|range|range_bits|cluster)'}
+KRE=${2:-'k_(num|sym)_(smem|range|range_bits|cluster|rankacc|rankcnt)'}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" || exit 1
 timeout 1500 python -m pytest tests/ -q -m gpu > gpurun_out/tests_$TAG.log 2>&1; tail -3 gpurun_out/tests_$TAG.log
