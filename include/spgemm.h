@@ -157,13 +157,18 @@ typedef enum {
     SPGEMM_OPT_BITMAP_RANK = 16,    /* 1 (default): CTA-per-row numeric groups order each row by a
                                        two-level bitmap rank over its column span;
                                        0: bucket sort (ablation) */
-    SPGEMM_OPT_RANK_ACC = 17        /* 1 (default): CTA-per-row numeric groups (4-9) accumulate each
+    SPGEMM_OPT_RANK_ACC = 17,       /* 1 (default): CTA-per-row numeric groups (4-9) accumulate each
                                        row directly at the rank of its column — the two-level
                                        bitmap over the row's span built first, used as a
                                        collision-free order-preserving hash;
                                        needs RANGE_HASH (column spans).  0: paper hash table +
                                        gather + rank; off while NUM_MIN_GROUP
                                        is forced */
+    SPGEMM_OPT_TINY = 18            /* 1 (default): numeric groups 0-1 run thread-per-row kernels
+                                       with the row's table in registers, kept in column order
+                                       (DESIGN.md §5.10); 2: symbolic groups 0-1 too (measured
+                                       slower than the partial-warp hash there); 0: the paper's
+                                       partial-warp hash groups.  Off while a MIN_GROUP is forced */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);
@@ -199,7 +204,8 @@ typedef enum {
     SPGEMM_KERNEL_RANGE = 3,    /* range rows: offset table, warp per row (kernels_range.cu)     */
     SPGEMM_KERNEL_CLUSTER = 4,  /* distributed shared-memory hash table (kernels_cluster.cu)     */
     SPGEMM_KERNEL_GLOBAL = 5,   /* global-memory hash table                  */
-    SPGEMM_KERNEL_RANK_BIG = 6  /* rank-indexed, level 2 in global memory, values reduced into C */
+    SPGEMM_KERNEL_RANK_BIG = 6, /* rank-indexed, level 2 in global memory, values reduced into C */
+    SPGEMM_KERNEL_TINY = 7      /* thread per row, sorted register table (kernels_tiny.cu)       */
 } spgemm_kernel_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);

@@ -25,11 +25,11 @@ OPTIONS = {
     "sym_min_group": 0, "num_min_group": 1, "sym_fill_limit": 2, "streams": 3,
     "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8, "range_hash": 9,
     "cluster": 10, "cluster_fill_limit": 11, "flat": 12, "graphs": 13, "range_warp": 14,
-    "range_min_nprod": 15, "bitmap_rank": 16, "rank_acc": 17,
+    "range_min_nprod": 15, "bitmap_rank": 16, "rank_acc": 17, "tiny": 18,
 }
 
 # spgemm_kernel_t (include/spgemm.h): kernel family that ran each group
-KERNELS = {0: "none", 1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big"}
+KERNELS = {0: "none", 1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big", 7: "tiny"}
 
 # Group ids of the range-row kernels (spgemm_internal.cuh kSymRange / kNumRange).
 SYM_RANGE_GROUP = 12

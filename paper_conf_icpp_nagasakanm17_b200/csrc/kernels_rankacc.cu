@@ -136,8 +136,8 @@ struct RankCfg {
 // the few rows above it take the re-walk path) — half the warps per row of KP*TPR = 2x the bound
 // (R-MAT s20: groups 6-8 1.86/2.21/1.90 -> 1.73/1.69/1.82 ms); group 5 keeps 128 threads (64:
 // the span-sized level-1 bitmap per CTA limits residency, 1.21 -> 1.38 ms)
-constexpr RankCfg kRankNum[] = {{0, 0, 0},   {0, 0, 0},   {0, 0, 0},   {64, 4, 2},  {64, 8, 2},
-                                {128, 8, 2}, {128, 8, 2}, {256, 8, 2}, {512, 8, 2}, {1024, 9, 2}};
+constexpr RankCfg kRankNum[] = {{0, 0, 0},   {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},
+                                {128, 8, 2}, {128, 12, 2}, {256, 12, 2}, {512, 12, 2}, {1024, 9, 2}};
 // symbolic groups 3-4 stay on the paper hash (faster there: measured R-MAT s20 0.28/0.66 ms vs
 // 0.53/0.69 ms); MC 4 measured slower than 2 for groups 5-8
 constexpr RankCfg kRankSym[] = {{0, 0, 0},    {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},
@@ -325,11 +325,12 @@ template <typename VT>
 constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 4 + (int)sizeof(BlockFlat<VT, 1024>); }
 
 // 40 registers (1536 threads per SM) for fp32 / symbolic; fp64 values need 64 (no spills)
-template <int TPR, int VB>
-constexpr int rank_min_blocks() { return TPR >= 1024 ? 1 : (VB > 4 ? 1024 : 1536) / TPR; }
+// (KP > 8 products per thread: 1280 threads, ~48 registers)
+template <int TPR, int VB, int KP = 8>
+constexpr int rank_min_blocks() { return TPR >= 1024 ? 1 : (VB > 4 ? 1024 : KP > 8 ? 1280 : 1536) / TPR; }
 
 template <typename VT, int TPR, long long UPPER, int KP, int MC>
-__global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT)>()) void k_num_rankacc(NumArgs a) {
+__global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT), KP>()) void k_num_rankacc(NumArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];

@@ -46,19 +46,52 @@ __device__ __forceinline__ int setup_glog(const int64_t* __restrict__ rpt, long 
 
 // Column range of every B row: bmm[k] = {min col, max col} ({INT_MAX, -1} if empty), and the
 // "some B row is not strictly increasing" flag.  G lanes per row (grid-stride over row blocks).
+constexpr int kDeferLen = 512;  // rows longer than this: one warp each in k_*_long
+
+// Warp-wide min/max and strictly-increasing check of B row [s0, s1), 8 loads (+8 predecessors)
+// in flight per lane.
+__device__ __forceinline__ void brow_warp(const int32_t* __restrict__ b_col, long long s0, long long s1, int lane,
+                                          int& mn, int& mx, bool& bad) {
+  int pmn = INT_MAX, pmx = -1;
+  bool pbad = false;
+  for (long long j = s0 + lane; j < s1; j += 8 * 32) {
+    int c[8], pv[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const long long q = j + 32 * u;
+      c[u] = q < s1 ? __ldg(b_col + q) : 0;
+      pv[u] = q < s1 && q > s0 ? __ldg(b_col + q - 1) : INT_MIN;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (j + 32 * u < s1) {
+        pmn = min(pmn, c[u]); pmx = max(pmx, c[u]);
+        pbad |= pv[u] != INT_MIN && c[u] <= pv[u];
+      }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
+    pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
+  }
+  mn = pmn; mx = pmx;
+  bad = __any_sync(0xffffffffu, pbad);
+}
+
 __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, const int64_t* __restrict__ b_rpt,
                                                                const int32_t* __restrict__ b_col,
-                                                               int2* __restrict__ bmm, int* __restrict__ unsorted) {
+                                                               int2* __restrict__ bmm, int* __restrict__ unsorted,
+                                                               int32_t* __restrict__ defer, int* __restrict__ ndefer) {
   const int glog = setup_glog(b_rpt, k);
   const int G = 1 << glog, lane = threadIdx.x & 31, gl = lane & (G - 1);
   const int rpc = kSetupThreads >> glog;
   bool bad = false;
-  // One lane per row (mean row length < 8, power-law shapes): rows interleaved over CTAs (row =
-  // base + slot * gridDim.x + blockIdx.x) — long rows cluster in index ranges, and contiguous
-  // slices hand one warp many of them in series (webbase: 152 -> 119 us; with G > 1 the
-  // contiguous slices' coalesced rpt loads win: cant 25 -> 31 us, R-MAT 241 -> 267 us interleaved)
+  // Contiguous row slices (coalesced rpt loads).  Rows longer than kDeferLen go to a list and are
+  // handled by k_*_long, one warp each: power-law generators cluster their hub rows, and a warp
+  // walking several of them in series set the kernel time (webbase: 152 us; interleaving rows
+  // over CTAs instead cost the short-row shapes their coalescing: cant 25 -> 31 us).
   const long long T = (long long)gridDim.x * rpc;
-  const bool ilv = G == 1;
+  constexpr bool ilv = false;
   for (long long base = 0; base < k; base += T) {
     const long long row = base + (ilv ? (long long)(threadIdx.x >> glog) * gridDim.x + blockIdx.x
                                       : (long long)blockIdx.x * rpc + (threadIdx.x >> glog));
@@ -99,34 +132,90 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, cons
       const int src = __ffs(longs) - 1;
       longs &= longs - 1;
       const long long s0 = __shfl_sync(0xffffffffu, b0, src), s1 = __shfl_sync(0xffffffffu, b1, src);
-      int pmn = INT_MAX, pmx = -1;
-      bool pbad = false;
-      for (long long j = s0 + lane; j < s1; j += 8 * 32) {  // 8 loads (+8 predecessors) in flight
-        int c[8], pv[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          const long long q = j + 32 * u;
-          c[u] = q < s1 ? __ldg(b_col + q) : 0;
-          pv[u] = q < s1 && q > s0 ? __ldg(b_col + q - 1) : INT_MIN;
-        }
-#pragma unroll
-        for (int u = 0; u < 8; ++u)
-          if (j + 32 * u < s1) {
-            pmn = min(pmn, c[u]); pmx = max(pmx, c[u]);
-            pbad |= pv[u] != INT_MIN && c[u] <= pv[u];
-          }
+      if (defer && s1 - s0 > kDeferLen) {  // warp-uniform: deferred to k_brow_minmax_long
+        if (lane == src) defer[atomicAdd(ndefer, 1)] = (int32_t)row;
+        continue;
       }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        pmn = min(pmn, __shfl_xor_sync(0xffffffffu, pmn, o));
-        pmx = max(pmx, __shfl_xor_sync(0xffffffffu, pmx, o));
-      }
-      bad |= __any_sync(0xffffffffu, pbad) && lane == src;
+      int pmn, pmx;
+      bool pbad;
+      brow_warp(b_col, s0, s1, lane, pmn, pmx, pbad);
+      bad |= pbad && lane == src;
       if (lane == src) { mn = pmn; mx = pmx; }
     }
-    if (row < k && gl == 0) bmm[row] = make_int2(mn, mx);
+    if (row < k && gl == 0 && !(defer && is_long && b1 - b0 > kDeferLen)) bmm[row] = make_int2(mn, mx);
   }
   if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(unsorted, 1);
+}
+
+// Deferred long B rows: one warp per row.
+__global__ __launch_bounds__(kSetupThreads) void k_brow_minmax_long(const int64_t* __restrict__ b_rpt,
+                                                                    const int32_t* __restrict__ b_col,
+                                                                    int2* __restrict__ bmm, int* __restrict__ unsorted,
+                                                                    const int32_t* __restrict__ defer,
+                                                                    const int* __restrict__ ndefer) {
+  const int lane = threadIdx.x & 31;
+  const int nw = gridDim.x * (kSetupThreads / 32);
+  const int n = *ndefer;
+  for (int i = blockIdx.x * (kSetupThreads / 32) + (threadIdx.x >> 5); i < n; i += nw) {
+    const int row = defer[i];
+    int mn, mx;
+    bool bad;
+    brow_warp(b_col, __ldg(b_rpt + row), __ldg(b_rpt + row + 1), lane, mn, mx, bad);
+    if (lane == 0) {
+      bmm[row] = make_int2(mn, mx);
+      if (bad) atomicOr(unsorted, 1);
+    }
+  }
+}
+
+// Warp-wide n_prod and column span of A row [s0, s1), 8 entries per lane in flight.
+__device__ __forceinline__ void nprod_warp(const int32_t* __restrict__ a_col, const int64_t* __restrict__ b_rpt,
+                                           const int2* __restrict__ bmm, long long s0, long long s1, int lane,
+                                           long long& np, int& lo, int& hi) {
+  long long part = 0;
+  int plo = INT_MAX, phi = -1;
+  for (long long j = s0 + lane; j < s1; j += 8 * 32) {
+    int kk[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) kk[u] = j + 32 * u < s1 ? __ldg(a_col + j + 32 * u) : -1;
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (kk[u] >= 0) {
+        part += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+        if (bmm) { const int2 r = __ldg(bmm + kk[u]); plo = min(plo, r.x); phi = max(phi, r.y); }
+      }
+  }
+  np = (long long)warp_sum_u64((unsigned long long)part);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    plo = min(plo, __shfl_xor_sync(0xffffffffu, plo, o));
+    phi = max(phi, __shfl_xor_sync(0xffffffffu, phi, o));
+  }
+  lo = plo; hi = phi;
+}
+
+// Row outputs of step (1)/(2): n_prod, span, group id (Table I bounds, or the range-row group).
+__device__ __forceinline__ int nprod_finish(long long row, long long np, int lo, int hi, int64_t* __restrict__ nprod,
+                                            int2* __restrict__ rlohi, uint8_t* __restrict__ grp,
+                                            int64_t* __restrict__ c_rpt, const Bounds& bd, bool b_ok, int& span_max) {
+  int g = -1;
+  nprod[row] = np;
+  if (rlohi) rlohi[row] = make_int2(lo, hi);
+  if (np == 0) {
+    c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
+  } else {
+    const long long R = (long long)hi - lo + 1;
+    // range rows (kernels_range.cu): narrow exact column span, enough products for a warp
+    if (b_ok && rlohi && np >= bd.range_min_np && np <= kRangeMaxNprod && R <= kRangeMaxSpan &&
+        R <= kRangeSpanPerProd * np) {
+      g = bd.range_group;
+      span_max = max(span_max, (int)R);
+    } else {
+      g = group_of(np, bd);
+    }
+  }
+  grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
+  return g;
 }
 
 // n_prod of every row (Alg. 2) with G lanes per row; also the column span [lo_i, hi_i] of row i
@@ -137,7 +226,7 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
     long long m, const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
     const int64_t* __restrict__ b_rpt, const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
     int2* __restrict__ rlohi, uint8_t* __restrict__ grp, int64_t* __restrict__ c_rpt,
-    DevAcc* __restrict__ acc, Bounds bd) {
+    DevAcc* __restrict__ acc, Bounds bd, int32_t* __restrict__ defer, int* __restrict__ ndefer) {
   __shared__ int s_cnt[kMaxGroups];
   __shared__ unsigned long long s_total, s_max;
   if (threadIdx.x < kMaxGroups) s_cnt[threadIdx.x] = 0;
@@ -149,8 +238,8 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
   const bool b_ok = bd.range_group >= 0 && __ldg(b_rpt + bd.range_k) < (1LL << 31);
   unsigned long long tot = 0, mxnp = 0;
   int span_max = 0;
-  const long long T = (long long)gridDim.x * rpc;  // rows interleaved over CTAs when G = 1 (see k_brow_minmax)
-  const bool ilv = G == 1;
+  const long long T = (long long)gridDim.x * rpc;  // contiguous slices, long rows deferred (see k_brow_minmax)
+  constexpr bool ilv = false;
   for (long long base = 0; base < m; base += T) {
     const long long row = base + (ilv ? (long long)(threadIdx.x >> glog) * gridDim.x + blockIdx.x
                                       : (long long)blockIdx.x * rpc + (threadIdx.x >> glog));
@@ -179,50 +268,27 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
       hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
     }
     unsigned longs = __ballot_sync(0xffffffffu, is_long && gl == 0);
+    bool deferred = false;
     while (longs) {
       const int src = __ffs(longs) - 1;
       longs &= longs - 1;
       const long long s0 = __shfl_sync(0xffffffffu, a0, src), s1 = __shfl_sync(0xffffffffu, a1, src);
-      long long part = 0;
-      int plo = INT_MAX, phi = -1;
-      for (long long j = s0 + lane; j < s1; j += 8 * 32) {  // 8 entries per lane in flight
-        int kk[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) kk[u] = j + 32 * u < s1 ? __ldg(a_col + j + 32 * u) : -1;
-#pragma unroll
-        for (int u = 0; u < 8; ++u)
-          if (kk[u] >= 0) {
-            part += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
-            if (bmm) { const int2 r = __ldg(bmm + kk[u]); plo = min(plo, r.x); phi = max(phi, r.y); }
-          }
+      if (defer && s1 - s0 > kDeferLen) {  // warp-uniform: deferred to k_nprod_long
+        if (lane == src) {
+          defer[atomicAdd(ndefer, 1)] = (int32_t)row;
+          deferred = true;
+        }
+        continue;
       }
-      part = (long long)warp_sum_u64((unsigned long long)part);
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        plo = min(plo, __shfl_xor_sync(0xffffffffu, plo, o));
-        phi = max(phi, __shfl_xor_sync(0xffffffffu, phi, o));
-      }
+      long long part;
+      int plo, phi;
+      nprod_warp(a_col, b_rpt, bmm, s0, s1, lane, part, plo, phi);
       if (lane == src) { np = part; lo = plo; hi = phi; }
     }
-    const bool lead = row < m && gl == 0;
+    const bool lead = row < m && gl == 0 && !deferred;
     int g = -1;
     if (lead) {
-      nprod[row] = np;
-      if (rlohi) rlohi[row] = make_int2(lo, hi);
-      if (np == 0) {
-        c_rpt[row + 1] = 0;  // reading R13: empty product row -> nnz 0, no kernel work
-      } else {
-        const long long R = (long long)hi - lo + 1;
-        // range rows (kernels_range.cu): narrow exact column span, enough products for a warp
-        if (b_ok && rlohi && np >= bd.range_min_np && np <= kRangeMaxNprod && R <= kRangeMaxSpan &&
-            R <= kRangeSpanPerProd * np) {
-          g = bd.range_group;
-          span_max = max(span_max, (int)R);
-        } else {
-          g = group_of(np, bd);
-        }
-      }
-      grp[row] = (uint8_t)(g < 0 ? 0xFF : g);
+      g = nprod_finish(row, np, lo, hi, nprod, rlohi, grp, c_rpt, bd, b_ok, span_max);
       tot += (unsigned long long)np;
       mxnp = max(mxnp, (unsigned long long)np);
     }
@@ -241,6 +307,37 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
   if (threadIdx.x == 0) {
     if (s_total) atomicAdd(&acc->total_nprod, s_total);
     if (s_max) atomicMax(&acc->max_nprod, s_max);
+  }
+}
+
+// Deferred long A rows of step (1)/(2): one warp per row, statistics straight to DevAcc.
+__global__ __launch_bounds__(kSetupThreads) void k_nprod_long(const int64_t* __restrict__ a_rpt,
+                                                              const int32_t* __restrict__ a_col,
+                                                              const int64_t* __restrict__ b_rpt,
+                                                              const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
+                                                              int2* __restrict__ rlohi, uint8_t* __restrict__ grp,
+                                                              int64_t* __restrict__ c_rpt, DevAcc* __restrict__ acc,
+                                                              Bounds bd, const int32_t* __restrict__ defer,
+                                                              const int* __restrict__ ndefer) {
+  const int lane = threadIdx.x & 31;
+  const int nw = gridDim.x * (kSetupThreads / 32);
+  const int n = *ndefer;
+  const bool b_ok = bd.range_group >= 0 && __ldg(b_rpt + bd.range_k) < (1LL << 31);
+  for (int i = blockIdx.x * (kSetupThreads / 32) + (threadIdx.x >> 5); i < n; i += nw) {
+    const int row = defer[i];
+    long long np;
+    int lo, hi;
+    nprod_warp(a_col, b_rpt, bmm, __ldg(a_rpt + row), __ldg(a_rpt + row + 1), lane, np, lo, hi);
+    if (lane == 0) {
+      int span_max = 0;
+      const int g = nprod_finish(row, np, lo, hi, nprod, rlohi, grp, c_rpt, bd, b_ok, span_max);
+      if (g >= 0) atomicAdd(&acc->sym_rows[g], 1ull);
+      if (np) {
+        atomicAdd(&acc->total_nprod, (unsigned long long)np);
+        atomicMax(&acc->max_nprod, (unsigned long long)np);
+      }
+      if (span_max > 0) atomicMax(&acc->range_rmax, span_max);
+    }
   }
 }
 
@@ -469,19 +566,27 @@ __global__ void k_splits(long long m, const int64_t* __restrict__ excl, int npar
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
                                const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
                                int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
-                               int* nlaunch) {
+                               int32_t* defer_a, int32_t* defer_b, int* nlaunch) {
   if (m == 0) return cudaSuccess;
   // grid-stride kernels: enough CTAs for any lanes-per-row choice (rows / 8 per CTA-pass at G = 32)
   auto grid_of = [](long long rows) {
     const long long want = (rows + (kSetupThreads / 32) - 1) / (kSetupThreads / 32);
     return (unsigned)(want < 148LL * 16 ? (want > 0 ? want : 1) : 148LL * 16);
   };
+  // deferred long rows (> kDeferLen entries): one warp each, 148 x 4 CTAs of 8 warps
+  const unsigned long_grid = 148 * 4;
   if (bmm && k > 0) {
-    k_brow_minmax<<<grid_of(k), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm, &acc->b_unsorted);
-    if (nlaunch) ++*nlaunch;
+    k_brow_minmax<<<grid_of(k), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm, &acc->b_unsorted, defer_b,
+                                                       &acc->defer_count[0]);
+    k_brow_minmax_long<<<long_grid, kSetupThreads, 0, s>>>(b_rpt, b_col, bmm, &acc->b_unsorted, defer_b,
+                                                           &acc->defer_count[0]);
+    if (nlaunch) *nlaunch += 2;
   }
-  k_nprod_group<<<grid_of(m), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b);
-  if (nlaunch) ++*nlaunch;
+  k_nprod_group<<<grid_of(m), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b,
+                                                     defer_a, &acc->defer_count[1]);
+  k_nprod_long<<<long_grid, kSetupThreads, 0, s>>>(a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b, defer_a,
+                                                   &acc->defer_count[1]);
+  if (nlaunch) *nlaunch += 2;
   return cudaGetLastError();
 }
 

@@ -87,8 +87,9 @@ struct spgemm_ctx {
   int timing = 1;
   int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
   long long range_min_np = kRangeMinNprodDefault;
-  int rank_acc = 1;
-  bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)      // CTA-per-row numeric groups: rank-indexed accumulation (kernels_rankacc.cu)
+  int rank_acc = 1;      // CTA-per-row groups: rank-indexed tables (kernels_rankacc.cu)
+  int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
+  bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)
   int bitmap_rank = 1;   // CTA-per-row numeric groups: two-level bitmap rank (else bucket sort)
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
@@ -99,6 +100,7 @@ struct spgemm_ctx {
   const int32_t *a_col = nullptr, *b_col = nullptr;
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
+  Buf defer_b;  // step (1): deferred long B rows (the A list reuses perm1, rewritten after sync 1)
   Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi, num_slab, num_slab_c,
       rbits, bbits;
   bool range_num = false;  // numeric range rows on for the last symbolic call (bitmap allocated, B sorted)
@@ -180,7 +182,8 @@ void release_state(spgemm_handle_t h) {
 
 void free_all(spgemm_handle_t h) {
   Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow,
-                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits, &h->bbits};
+                &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits, &h->bbits,
+                &h->defer_b};
   for (Buf* b : all) buf_free(h, *b);
   release_state(h);
 }
@@ -519,6 +522,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->range_min_np = v; break;
     case SPGEMM_OPT_BITMAP_RANK: h->bitmap_rank = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_ACC: h->rank_acc = v ? 1 : 0; break;
+    case SPGEMM_OPT_TINY:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "TINY must be 0, 1 or 2");
+      h->tiny = (int)v; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -573,6 +579,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   if (h->range_hash) {
     ALLOC(h->bmm, sizeof(int2) * std::max<int64_t>(k, 1));
     ALLOC(h->rlohi, sizeof(int2) * m);
+    ALLOC(h->defer_b, sizeof(int32_t) * std::max<int64_t>(k, 1));
   }
   if (h->timing) CK(cudaEventRecord(h->ev[0], h->stream));
   if (h->validate) {
@@ -584,7 +591,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
     int nl = 0;
     CK(launch_nprod_group(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, static_cast<int2*>(h->bmm.p),
                           static_cast<int64_t*>(h->nprod.p), static_cast<int2*>(h->rlohi.p),
-                          static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h), &nl));
+                          static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h),
+                          static_cast<int32_t*>(h->perm1.p), static_cast<int32_t*>(h->defer_b.p), &nl));
     launches += nl;
   }
   CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
@@ -669,7 +677,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
-                                 (long long)h->rank_acc};
+                                 (long long)h->rank_acc, (long long)h->tiny};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -696,9 +704,11 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       SymArgs ga = sa;
       ga.rows = perm1 + off1.off[g];
       ga.nrows = rows;
-      if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
+      const bool tiny_g = h->tiny >= 2 && h->sym_min_group < 0 && g <= 1;  // measured slower than the hash
+      if (tiny_g) CK(launch_symbolic_tiny(s, g, ga));
+      else if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
       else CK(launch_symbolic_group(s, g, ga, h->num_sms));
-      h->gkind[0][g] = rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
+      h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
       ++launches;
       if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
         SymArgs gb = sa;
@@ -912,7 +922,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     // numeric re-runs with new values of the same structure, or repeated multiplies)
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, btotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
-                                   h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc,
+                                   h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
@@ -989,7 +999,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(cudaMalloc(&ga.prof, sizeof(unsigned long long) * 4 * rows));
             CK(cudaMemset(ga.prof, 0, sizeof(unsigned long long) * 4 * rows));
           }
-          if (rank_acc_on(g)) {
+          if (h->tiny && h->num_min_group < 0 && g <= 1) {
+            CK(launch_numeric_tiny(st, g, fp64, ga));
+            h->gkind[1][g] = SPGEMM_KERNEL_TINY;
+          } else if (rank_acc_on(g)) {
             NumArgs ra = ga;
             ra.l1_words = l1w_rank;
             CK(launch_numeric_rankacc(st, g, fp64, ra));

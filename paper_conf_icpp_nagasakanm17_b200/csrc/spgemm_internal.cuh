@@ -115,6 +115,7 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   int cursor[2][kMaxGroups];
   int range_rmax;  // max column span R_i over the range rows (sizes the per-warp tables)
   int row_counter[4];  // numeric cluster groups: dynamic row counters (zeroed per numeric call)
+  int defer_count[2];  // step (1): deferred long rows of B (0) and A (1)
 };
 
 struct Bounds {  // group bounds passed by value
@@ -759,7 +760,7 @@ __device__ __forceinline__ unsigned long long gtimer() {
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
                                const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
                                int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
-                               int* nlaunch);
+                               int32_t* defer_a, int32_t* defer_b, int* nlaunch);
 cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1, const uint8_t* grp2,
                                const int64_t* nprod, const int64_t* a_rpt, const int64_t* c_rpt, DevAcc* acc);
 cudaError_t launch_group_scatter(cudaStream_t s, long long m, const uint8_t* grp, Offsets off,
@@ -783,6 +784,8 @@ int rankacc_smem_bytes(int group, bool fp64, int l1_words);
 cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a);
 int rankcnt_smem_bytes(int group, int l1_words);
 cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
+cudaError_t launch_symbolic_tiny(cudaStream_t s, int group, const SymArgs& a);
+cudaError_t launch_numeric_tiny(cudaStream_t s, int group, bool fp64, const NumArgs& a);
 int rankbig_smem_bytes(bool fp64, int l1_words);
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows);

@@ -97,3 +97,25 @@ def test_product_path_has_no_oracle_import():
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "gustavson" not in txt.lower(), f
+
+
+def test_binding_matches_header_enums_and_stats_layout(tmp_path):
+    """The Python binding's option ids, kernel-family ids and spgemm_stats_t layout agree with
+    include/spgemm.h (compiled with gcc: sizeof and offsetof of every field)."""
+    import subprocess
+    from paper_conf_icpp_nagasakanm17_b200 import _lib
+    txt = open(HEADER).read()
+    opts = {m.group(1).lower(): int(m.group(2)) for m in re.finditer(r"SPGEMM_OPT_(\w+)\s*=\s*(\d+)", txt)}
+    assert opts == _lib.OPTIONS
+    kinds = {int(m.group(2)): m.group(1).lower() for m in re.finditer(r"SPGEMM_KERNEL_(\w+)\s*=\s*(\d+)", txt)}
+    assert kinds == _lib.KERNELS
+    fields = [f for f, _ in _lib.Stats._fields_]
+    src = tmp_path / "layout.c"
+    src.write_text("#include <stdio.h>\n#include <stddef.h>\n#include \"spgemm.h\"\nint main(void){\n"
+                   "printf(\"%zu\\n\", sizeof(spgemm_stats_t));\n" +
+                   "".join(f"printf(\"%zu\\n\", offsetof(spgemm_stats_t, {f}));\n" for f in fields) + "return 0;}\n")
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c99", f"-I{os.path.dirname(HEADER)}", str(src), "-o", str(exe)])
+    out = [int(x) for x in subprocess.check_output([str(exe)]).split()]
+    assert out[0] == ctypes.sizeof(_lib.Stats)
+    assert out[1:] == [getattr(_lib.Stats, f).offset for f in fields]
