@@ -271,14 +271,16 @@ __global__ __launch_bounds__(1024, 1) void k_sym_range(SymArgs a, int rcap) {
 // rows wider than the range rows' R_max are never read.)  One warp per B row.
 __global__ __launch_bounds__(256) void k_brow_bits(long long k, const int64_t* __restrict__ b_rpt,
                                                    const int32_t* __restrict__ b_col, const int2* __restrict__ bmm,
-                                                   unsigned* __restrict__ bbits, int bw) {
+                                                   unsigned* __restrict__ bbits, int bw, int* __restrict__ wmax) {
   __shared__ unsigned s_w[8][64];
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   unsigned* sw = s_w[wi];
+  int my_wmax = 0;
   for (long long row = (long long)blockIdx.x * 8 + wi; row < k; row += (long long)gridDim.x * 8) {
     const int2 mm = __ldg(bmm + row);
     if (mm.y < mm.x || (long long)mm.y - mm.x + 1 > 32LL * bw) continue;  // empty or too wide: unused
     const int nw = (mm.y - mm.x) / 32 + 1;
+    my_wmax = max(my_wmax, nw);
     for (int w = lane; w < nw; w += 32) sw[w] = 0u;
     __syncwarp();
     const long long b0 = __ldg(b_rpt + row), b1 = __ldg(b_rpt + row + 1);
@@ -290,6 +292,7 @@ __global__ __launch_bounds__(256) void k_brow_bits(long long k, const int64_t* _
     for (int w = lane; w < nw; w += 32) bbits[row * bw + w] = sw[w];
     __syncwarp();
   }
+  if (lane == 0 && my_wmax > 0) atomicMax(wmax, my_wmax);
 }
 
 // Step (3) on range rows with R_max <= 1024, from the B-row bitmaps: the pattern of row i is the
@@ -298,19 +301,77 @@ __global__ __launch_bounds__(256) void k_brow_bits(long long k, const int64_t* _
 // Lane gl of a group of L = 32/H lanes owns output word gl; H A non-zeros are OR-ed at a time (H
 // groups, L >= words of the row), the groups are OR-reduced at the end.  Writes nnz_i = popcount
 // and the pattern bitmap (the numeric gather's input).
+//
+// When every B bitmap has <= 31 words (wmax, from k_brow_bits), the OR is done per A non-zero
+// instead: LB = next_pow2(wmax + 1) lanes per non-zero (lane g produces output word q + g from B
+// words g and g-1), 32/LB non-zeros per step, OR-ed into a per-warp shared row bitmap — fewer
+// steps than owning all output words per lane group (cant: 5-word B rows in 9-word output rows:
+// 4 non-zeros per step instead of 2).
 __global__ __launch_bounds__(1024, 1) void k_sym_range_bits(SymArgs a, const unsigned* __restrict__ bbits, int bw,
-                                                            const int2* __restrict__ bmm) {
+                                                            const int2* __restrict__ bmm, const int* __restrict__ wmax) {
   __shared__ int4 s_meta[32][kMetaBatch];  // (B bitmap offset lo, hi, shift, words)
+  __shared__ unsigned s_row[32][32];       // per-warp row bitmap (per-non-zero mode)
   __shared__ int s_next;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   int4* meta = s_meta[w];
+  unsigned* rowb = s_row[w];
   const unsigned mb = smem_u32(meta);
+  const int wm = *wmax;
+  const int lblog = wm + 1 <= 2 ? 1 : wm + 1 <= 4 ? 2 : wm + 1 <= 8 ? 3 : wm + 1 <= 16 ? 4 : 5;
+  const bool per_nz = wm + 1 <= 16;  // else the output-word-owner loop below
   const RowQueue rq = row_queue(a.nrows, &s_next);
   for (long long r = rq.pop(lane); r >= 0; r = rq.pop(lane)) {
     const int row = a.rows[r];
     const int2 rr = __ldg(a.rlohi + row);
     const int lo = rr.x, R = rr.y - rr.x + 1;  // R <= 1024
     const int nw = (R + 31) >> 5;
+    if (per_nz) {
+      const int LB = 1 << lblog, g = lane & (LB - 1), hh = lane >> lblog, H = 32 >> lblog;
+      if (lane < nw) rowb[lane] = 0u;
+      const long long a0 = __ldg(a.a_rpt + row);
+      const int na = (int)(__ldg(a.a_rpt + row + 1) - a0);
+      const int32_t* __restrict__ ac = a.a_col + a0;
+      for (int bb = 0; bb < na; bb += kMetaBatch) {
+        const int j = bb + lane;
+        int4 m = make_int4(0, 0, 0, 0);
+        if (j < na) {
+          const int kk = __ldg(ac + j);
+          const int2 mm = __ldg(bmm + kk);
+          if (mm.y >= mm.x) {
+            const long long off = (long long)kk * bw;
+            m = make_int4((int)(off & 0xffffffff), (int)(off >> 32), mm.x - lo, (mm.y - mm.x) / 32 + 1);
+          }
+        }
+        meta[lane] = m;
+        __syncwarp();
+        const int cnt = min(kMetaBatch, na - bb);
+#pragma unroll 1
+        for (int e0 = 0; e0 < cnt; e0 += H) {
+          const int e = e0 + hh;
+          int4 me = make_int4(0, 0, 0, 0);
+          if (e < cnt) asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                                    : "=r"(me.x), "=r"(me.y), "=r"(me.z), "=r"(me.w) : "r"(mb + 16u * e));
+          const int q = me.z >> 5, sh = me.z & 31;
+          const unsigned* bk = bbits + (((long long)me.y << 32) | (unsigned)me.x);
+          const unsigned x = g < me.w ? __ldg(bk + g) : 0u;
+          unsigned y = __shfl_up_sync(0xffffffffu, x, 1, LB);
+          if (g == 0) y = 0u;
+          const unsigned v = (x << sh) | (sh ? (y >> (32 - sh)) : 0u);
+          if (v) atomicOr(rowb + q + g, v);
+        }
+        __syncwarp();
+      }
+      int cnt = 0;
+      if (lane < nw) {
+        const unsigned acc = rowb[lane];
+        if (a.rbits) a.rbits[r * a.rwcap + lane] = acc;
+        cnt = __popc(acc);
+      }
+      cnt = __reduce_add_sync(0xffffffffu, cnt);
+      if (lane == 0) a.c_cnt[row] = cnt;
+      __syncwarp();
+      continue;
+    }
     const int hlog = nw <= 8 ? 2 : (nw <= 16 ? 1 : 0);  // H = 1 << hlog A non-zeros at a time
     const int L = 32 >> hlog, gl = lane & (L - 1), h = lane >> (5 - hlog);
     const long long a0 = __ldg(a.a_rpt + row);
@@ -482,19 +543,19 @@ cudaError_t launch_symbolic_range(cudaStream_t s, const SymArgs& a, int rmax, in
 }
 
 cudaError_t launch_brow_bits(cudaStream_t s, long long k, const int64_t* b_rpt, const int32_t* b_col,
-                             const int2* bmm, unsigned* bbits, int bw, int num_sms) {
+                             const int2* bmm, unsigned* bbits, int bw, int* wmax, int num_sms) {
   if (k <= 0) return cudaSuccess;
   const long long want = (k + 7) / 8;
   const long long cap = (long long)num_sms * 8;
-  k_brow_bits<<<(unsigned)(want < cap ? want : cap), 256, 0, s>>>(k, b_rpt, b_col, bmm, bbits, bw);
+  k_brow_bits<<<(unsigned)(want < cap ? want : cap), 256, 0, s>>>(k, b_rpt, b_col, bmm, bbits, bw, wmax);
   return cudaGetLastError();
 }
 
 cudaError_t launch_symbolic_range_bits(cudaStream_t s, const SymArgs& a, const unsigned* bbits, int bw,
-                                       const int2* bmm, int num_sms) {
+                                       const int2* bmm, const int* wmax, int num_sms) {
   if (a.nrows <= 0) return cudaSuccess;
   const int grid = range_grid(k_sym_range_bits, 1024, 0, num_sms, a.nrows, 32);
-  k_sym_range_bits<<<grid, 1024, 0, s>>>(a, bbits, bw, bmm);
+  k_sym_range_bits<<<grid, 1024, 0, s>>>(a, bbits, bw, bmm, wmax);
   return cudaGetLastError();
 }
 

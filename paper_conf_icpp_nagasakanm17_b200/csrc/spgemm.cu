@@ -743,9 +743,9 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       ra.nrows = (long long)h->snap1.sym_rows[kSymRange];
       if (range_bw > 0) {  // B-row bitmaps, then the bitmap-union count
         CK(launch_brow_bits(s, k, b_rpt, b_col, static_cast<const int2*>(h->bmm.p), static_cast<unsigned*>(h->bbits.p),
-                            range_bw, h->num_sms));
+                            range_bw, &dacc->bbits_wmax, h->num_sms));
         CK(launch_symbolic_range_bits(s, ra, static_cast<const unsigned*>(h->bbits.p), range_bw,
-                                      static_cast<const int2*>(h->bmm.p), h->num_sms));
+                                      static_cast<const int2*>(h->bmm.p), &dacc->bbits_wmax, h->num_sms));
         launches += 2;
       } else {
         CK(launch_symbolic_range(s, ra, h->snap1.range_rmax, h->num_sms));

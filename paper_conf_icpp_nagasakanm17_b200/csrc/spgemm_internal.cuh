@@ -116,6 +116,7 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   int range_rmax;  // max column span R_i over the range rows (sizes the per-warp tables)
   int row_counter[4];  // numeric cluster groups: dynamic row counters (zeroed per numeric call)
   int defer_count[2];  // step (1): deferred long rows of B (0) and A (1)
+  int bbits_wmax;      // range rows: max words of a B-row bitmap (k_brow_bits)
 };
 
 struct Bounds {  // group bounds passed by value
@@ -793,9 +794,9 @@ cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumA
 cudaError_t launch_symbolic_range(cudaStream_t s, const SymArgs& a, int rmax, int num_sms);
 cudaError_t launch_numeric_range(cudaStream_t s, bool fp64, const NumArgs& a, int rmax, int num_sms);
 cudaError_t launch_brow_bits(cudaStream_t s, long long k, const int64_t* b_rpt, const int32_t* b_col,
-                             const int2* bmm, unsigned* bbits, int bw, int num_sms);
+                             const int2* bmm, unsigned* bbits, int bw, int* wmax, int num_sms);
 cudaError_t launch_symbolic_range_bits(cudaStream_t s, const SymArgs& a, const unsigned* bbits, int bw,
-                                       const int2* bmm, int num_sms);
+                                       const int2* bmm, const int* wmax, int num_sms);
 int range_warps(long long per_warp);
 int range_rcap(long long rmax);
 int range_wcap(long long rmax);
