@@ -31,6 +31,8 @@
 // 93-98% on cant, vs 36% for the CTA-per-row groups).  Per-warp tables are R_cap (= max R_i of
 // the group) slots, so shared memory does not limit occupancy the way the n_prod-sized tables of
 // Table I do.
+#include <cstdlib>
+
 #include "spgemm_internal.cuh"
 
 namespace spg {
@@ -519,7 +521,11 @@ cudaError_t set_smem(K kernel, size_t smem, size_t& configured) {
 
 // Warps per CTA for a per-warp table of `per_warp` bytes: <= 32, <= kRangeSmemBudget in total.
 int range_warps(long long per_warp) {
-  long long w = per_warp > 0 ? kRangeSmemBudget / per_warp : 32;
+  static const long long budget = [] {
+    const char* e = getenv("SPGEMM_RANGE_BUDGET");  // diagnostics: per-CTA table budget (bytes)
+    return e ? atoll(e) : kRangeSmemBudget;
+  }();
+  long long w = per_warp > 0 ? budget / per_warp : 32;
   if (w > 32) w = 32;
   if (w < 1) w = 1;
   return (int)w;
