@@ -797,7 +797,7 @@ cudaError_t launch_brow_bits(cudaStream_t s, long long k, const int64_t* b_rpt, 
                              const int2* bmm, unsigned* bbits, int bw, int* wmax, int num_sms);
 cudaError_t launch_symbolic_range_bits(cudaStream_t s, const SymArgs& a, const unsigned* bbits, int bw,
                                        const int2* bmm, const int* wmax, int num_sms);
-int range_warps(long long per_warp);
+int range_warps(long long per_warp, long long budget_default = kRangeSmemBudget);
 int range_rcap(long long rmax);
 int range_wcap(long long rmax);
 int cluster_capacity_sym();
