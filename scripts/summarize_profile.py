@@ -77,7 +77,7 @@ def launches():
             out.append((int(d["ID"]), d["Kernel Name"], float(d["Metric Value"]) / 1e3))
     # one bench step = the launches between two k_brow_minmax (first kernel of a step)
     starts = [i for i, (_, k, _) in enumerate(out) if "k_brow_minmax" in k or "k_nprod_group" in k and "k_brow" not in k]
-    starts = [i for i, (_, k, _) in enumerate(out) if "k_brow_minmax" in k] or starts
+    starts = [i for i, (_, k, _) in enumerate(out) if re.search(r"k_brow_minmax(?!_)", k)] or starts
     step = out[starts[-2]:starts[-1]] if len(starts) >= 2 else out
     tot = sum(t for _, k, t in step if k.startswith(("void spg", "spg")))
     lines = [f"# ncu launch list ({TAG}) — one bench step of `python bench.py` (cant-like A^2, fp32)", "",
