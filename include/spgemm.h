@@ -154,9 +154,11 @@ typedef enum {
                                        0: Table-I groups only.  Needs RANGE_HASH; off while a
                                        MIN_GROUP is forced */
     SPGEMM_OPT_RANGE_MIN_NPROD = 15,/* n_prod lower bound of range rows (default 256) */
-    SPGEMM_OPT_BITMAP_RANK = 16,    /* 1 (default): CTA-per-row numeric groups order each row by a
-                                       two-level bitmap rank over its column span;
-                                       0: bucket sort (ablation) */
+    SPGEMM_OPT_BITMAP_RANK = 16,    /* CTA-per-row numeric hash groups order each row by a
+                                       two-level bitmap rank over its column span:
+                                       1 (default) where the level-1 width n/1024 + 1 is at most
+                                       the group's nnz bound, else bucket sort; 2: always;
+                                       0: bucket sort everywhere (ablation) */
     SPGEMM_OPT_RANK_ACC = 17,       /* 1 (default): CTA-per-row numeric groups (4-9) accumulate each
                                        row directly at the rank of its column — the two-level
                                        bitmap over the row's span built first, used as a
@@ -164,11 +166,19 @@ typedef enum {
                                        needs RANGE_HASH (column spans).  0: paper hash table +
                                        gather + rank; off while NUM_MIN_GROUP
                                        is forced */
-    SPGEMM_OPT_TINY = 18            /* 1 (default): numeric groups 0-1 run thread-per-row kernels
+    SPGEMM_OPT_TINY = 18,           /* 1 (default): numeric groups 0-1 run thread-per-row kernels
                                        with the row's table in registers, kept in column order
                                        (DESIGN.md §5.10); 2: symbolic groups 0-1 too (measured
                                        slower than the partial-warp hash there); 0: the paper's
                                        partial-warp hash groups.  Off while a MIN_GROUP is forced */
+    SPGEMM_OPT_RANK_L1_PCT = 19,    /* numeric rank kernels (RANK_ACC) only for groups whose nnz
+                                       bound B satisfies 100 * W <= v * B, W = level-1 bitmap
+                                       words of the column range (n / 1024 + 1): wide matrices
+                                       keep the paper hash on their small-row groups (the level-1
+                                       clear + prefix costs more than the row).  Default 500,
+                                       0 = no limit */
+    SPGEMM_OPT_RANK_L1_PCT_SYM = 20 /* same for the symbolic rank-count kernels, B = the group's
+                                       n_prod bound.  Default 150, 0 = no limit */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

@@ -89,9 +89,17 @@ struct spgemm_ctx {
   int range_warp = 1;    // warp-per-row kernels for range rows (kernels_range.cu)
   long long range_min_np = kRangeMinNprodDefault;
   int rank_acc = 1;      // CTA-per-row groups: rank-indexed tables (kernels_rankacc.cu)
+  // rank kernels only for groups with 100 * level-1 words <= pct * group key bound (0: always);
+  // R-MAT s22 (4097 words), rank vs paper hash + bucket sort: numeric group 4 (bound 256) 11.6 vs
+  // 4.1 ms, group 5 (512) 13.5 vs 9.0, group 6 (1024) 14.6 vs 17.8; symbolic group 6 (2048) 6.7
+  // vs 4.5, group 7 (4096) 3.6 vs 4.6
+  long long rank_l1_pct = 500, rank_l1_pct_sym = 150;
   int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
   bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)
-  int bitmap_rank = 1;   // CTA-per-row numeric groups: two-level bitmap rank (else bucket sort)
+  // CTA-per-row numeric hash groups: two-level bitmap rank (else bucket sort); 1 = only where the
+  // level-1 width W <= the group's nnz bound (R-MAT s22, W = 4097: bucket 4.1 ms vs bitmap 21.9 ms
+  // on group 4, 25.4 vs 28.5 on group 7), 2 = always
+  int bitmap_rank = 1;
   long long ws_budget = 8LL << 30;
   // state of the last symbolic call
   int state = 0;
@@ -528,8 +536,16 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_RANGE_MIN_NPROD:
       if (v < 1 || v > kRangeMaxNprod) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANGE_MIN_NPROD out of range");
       h->range_min_np = v; break;
-    case SPGEMM_OPT_BITMAP_RANK: h->bitmap_rank = v ? 1 : 0; break;
+    case SPGEMM_OPT_BITMAP_RANK:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "BITMAP_RANK must be 0, 1 or 2");
+      h->bitmap_rank = (int)v; break;
     case SPGEMM_OPT_RANK_ACC: h->rank_acc = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_L1_PCT:
+      if (v < 0 || v > (1LL << 40)) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_L1_PCT out of range");
+      h->rank_l1_pct = v; break;
+    case SPGEMM_OPT_RANK_L1_PCT_SYM:
+      if (v < 0 || v > (1LL << 40)) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_L1_PCT_SYM out of range");
+      h->rank_l1_pct_sym = v; break;
     case SPGEMM_OPT_TINY:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "TINY must be 0, 1 or 2");
       h->tiny = (int)v; break;
@@ -655,7 +671,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   // rank-count kernels for the CTA-per-row groups (kernels_rankacc.cu; needs the column spans)
   auto rank_cnt_on = [&](int g) {
     return h->rank_acc && h->rlohi.p != nullptr && h->sym_min_group < 0 && g >= 5 && g <= 9 &&
-           rankcnt_smem_bytes(g, sa.l1_words) <= kSmemLimit;
+           rankcnt_smem_bytes(g, sa.l1_words) <= kSmemLimit &&
+           (h->rank_l1_pct_sym == 0 || 100LL * sa.l1_words <= h->rank_l1_pct_sym * kSymGroups[g].upper);
   };
   // range rows: pattern bitmap (symbolic -> numeric gather), rwcap words per row of the group
   const long long n_range = (long long)h->snap1.sym_rows[kSymRange];
@@ -685,7 +702,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
-                                 (long long)h->rank_acc, (long long)h->tiny};
+                                 (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -885,7 +902,8 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const bool low_compression = (double)h->snap1.total_nprod <= 2.5 * (double)h->nnzc;
     auto rank_acc_on = [&](int g) {
       return h->rank_acc && low_compression && h->rlohi.p != nullptr && h->num_min_group < 0 && g >= 3 && g <= 9 &&
-             rankacc_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit;
+             rankacc_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit &&
+             (h->rank_l1_pct == 0 || 100LL * l1w_rank <= h->rank_l1_pct * kNumGroups[g].upper);
     };
     // cluster groups (clusters of 2/4/8 CTAs): bitmap + prefix scratch per resident cluster
     const long long cwords = h->n / 32 + 2;
@@ -931,7 +949,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, btotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
-                                   (long long)low_compression};
+                                   (long long)low_compression, h->rank_l1_pct};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
@@ -1016,7 +1034,9 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(launch_numeric_rankacc(st, g, fp64, ra));
             h->gkind[1][g] = SPGEMM_KERNEL_RANK;
           } else {
-            CK(launch_numeric_group(st, g, fp64, ga));
+            NumArgs hb = ga;
+            if (h->bitmap_rank == 1 && g < kNumNumBounds && (long long)hb.l1_words > kNumGroups[g].upper) hb.l1_words = 0;
+            CK(launch_numeric_group(st, g, fp64, hb));
             h->gkind[1][g] = SPGEMM_KERNEL_HASH;
           }
           if (ga.prof) {

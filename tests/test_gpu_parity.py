@@ -136,7 +136,7 @@ def test_forced_symbolic_group(spg, group, range_hash):
 
 @pytest.mark.parametrize("range_hash", [0, 1])
 @pytest.mark.parametrize("group", list(range(0, 14)))
-@pytest.mark.parametrize("bitmap_rank", [1, 0])  # CTA groups: two-level bitmap rank / bucket sort
+@pytest.mark.parametrize("bitmap_rank", [2, 0])  # CTA groups: two-level bitmap rank / bucket sort
 def test_forced_numeric_group(spg, group, range_hash, bitmap_rank):
     if bitmap_rank == 0 and not 4 <= group <= 9:
         pytest.skip("bucket sort ablation only differs in the CTA-per-row groups")
@@ -565,6 +565,28 @@ def test_rank_acc_vs_paper_hash(spg, name, dtype):
             assert st["sym_kernel"][g] == 2, (g, st["sym_kernel"])
     got = check(spg, A, A, dtype, opts={"rank_acc": 0}, what=f"{name} paper hash")
     assert all(k in (0, 1, 3, 4, 5, 7) for k in got[3]["num_kernel"][:13]), got[3]["num_kernel"]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_rank_l1_pct_splits_groups(spg, dtype):
+    """RANK_L1_PCT: the rank kernels run only for groups whose key bound B has 100*W <= v*B
+    (W = n/1024 + 1 level-1 words); the groups below keep the paper hash, results unchanged."""
+    A = synth.rmat(14).with_values("uniform", 9)
+    w = A.n // 1024 + 1
+    got = check(spg, A, A, dtype, opts={"rank_l1_pct": 1, "rank_l1_pct_sym": 1}, what="rank_l1_pct=1")
+    st = got[3]
+    num_bounds = [8, 16, 64, 128, 256, 512, 1024, 2048, 4096, 8192]
+    sym_bounds = [16, 32, 128, 256, 512, 1024, 2048, 4096, 8192, 16384]
+    seen = set()
+    for g in range(3, 10):
+        if st["num_rows"][g]:
+            want = 2 if 100 * w <= num_bounds[g] else 1
+            seen.add(want)
+            assert st["num_kernel"][g] == want, (g, st["num_kernel"])
+    for g in range(5, 10):
+        if st["sym_rows"][g]:
+            assert st["sym_kernel"][g] == (2 if 100 * w <= sym_bounds[g] else 1), (g, st["sym_kernel"])
+    assert 1 in seen, "no CTA group fell back to the paper hash"
 
 
 @pytest.mark.parametrize("name", ["rmat14", "mixed:qcd"])
