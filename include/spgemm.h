@@ -119,7 +119,7 @@ typedef enum {
                                        last group index = global-memory fallback */
     SPGEMM_OPT_NUM_MIN_GROUP = 1,   /* same for the numeric grouping */
     SPGEMM_OPT_SYM_FILL_LIMIT = 2,  /* optimistic shared-memory table: abort a row after v
-                                       distinct keys (default table/2) */
+                                       distinct keys (default 3/4 of the table) */
     SPGEMM_OPT_STREAMS = 3,         /* 1 = one stream per group, 0 = serial */
     SPGEMM_OPT_VALIDATE = 4,        /* 1 = O(nnz) input validation in spgemm_symbolic */
     SPGEMM_OPT_LANES = 5,           /* lanes per B row (power of two 1..32), 0 = auto */
