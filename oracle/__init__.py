@@ -6,6 +6,9 @@ it and shares no code with it.  Arithmetic lives in oracle/gustavson.c (plain C,
 row-wise Gustavson, Alg. 1 and PAPER.md:90-96 Alg. 2) and
 oracle/binning.py (Table-I style grouping).
 
+Row-parallel variants (symbolic_omp, spgemm(parallel=True)): SURVEY.md §8(c) step 6, each row
+still summed in Algorithm 1 order; pinned to the single-thread functions bit for bit.
+
 Pins: tests/test_oracle_pins.py (closed forms, paper-printed Table II QCD count,
 identities, brute force, column unions, scipy cross-check).  "parity unpinned": none of
 the functions below.
@@ -26,7 +29,7 @@ _SRC = os.path.join(_HERE, "gustavson.c")
 _SO = os.path.join(_HERE, "liboracle.so")
 _LIB = None
 
-CC_FLAGS = ["-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-shared", "-fPIC"]
+CC_FLAGS = ["-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC"]
 
 
 def build(force: bool = False) -> str:
@@ -46,9 +49,13 @@ def _lib():
         lib.oracle_nprod.argtypes = [I64, P, P, P, P]
         lib.oracle_symbolic.restype = ctypes.c_int
         lib.oracle_symbolic.argtypes = [I64, I64, I64, P, P, P, P, P]
-        for f in (lib.oracle_numeric_f64, lib.oracle_numeric_f32):
+        lib.oracle_symbolic_omp.restype = ctypes.c_int
+        lib.oracle_symbolic_omp.argtypes = [I64, I64, I64, P, P, P, P, P]
+        for f in (lib.oracle_numeric_f64, lib.oracle_numeric_f32, lib.oracle_numeric_omp_f64,
+                  lib.oracle_numeric_omp_f32):
             f.restype = ctypes.c_int
             f.argtypes = [I64, I64, I64, P, P, P, P, P, P, P, P, P, P]
+        lib.oracle_threads.restype = ctypes.c_int
         _LIB = lib
     return _LIB
 
@@ -83,22 +90,47 @@ def symbolic(A, B) -> np.ndarray:
     return c_rpt
 
 
-def spgemm(A, B, dtype=np.float64):
+def symbolic_omp(A, B) -> np.ndarray:
+    """symbolic() on all host cores (row-parallel; identical result)."""
+    a_rpt, a_col = _csr_arrays(A)
+    b_rpt, b_col = _csr_arrays(B)
+    c_rpt = np.empty(A.m + 1, dtype=np.int64)
+    rc = _lib().oracle_symbolic_omp(A.m, B.m, B.n, _p(a_rpt), _p(a_col), _p(b_rpt), _p(b_col), _p(c_rpt))
+    if rc != 0:
+        raise ValueError(f"oracle_symbolic_omp failed: {rc}")
+    return c_rpt
+
+
+def threads() -> int:
+    """Threads the row-parallel functions use (OMP_NUM_THREADS, else all cores of the process)."""
+    return int(_lib().oracle_threads())
+
+
+def cores() -> int:
+    """Host cores available to this process."""
+    return len(os.sched_getaffinity(0))
+
+
+def spgemm(A, B, dtype=np.float64, parallel: bool = False, with_abs: bool = True):
     """C = A*B in working precision `dtype` (np.float32 or np.float64).
 
-    Returns (rpt int64[m+1], col int32[nnz], val dtype[nnz], absval float64[nnz]) where
-    absval = (|A|*|B|)_ij is the scale of the comparison tolerance."""
+    Returns (rpt int64[m+1], col int32[nnz], val dtype[nnz], absval float64[nnz] or None) where
+    absval = (|A|*|B|)_ij is the scale of the comparison tolerance.  parallel=True runs the
+    row-parallel functions (same result, all host cores)."""
     dtype = np.dtype(dtype)
     a_rpt, a_col = _csr_arrays(A)
     b_rpt, b_col = _csr_arrays(B)
     a_val = np.ascontiguousarray(A.val, dtype=dtype)
     b_val = np.ascontiguousarray(B.val, dtype=dtype)
-    c_rpt = symbolic(A, B)
+    c_rpt = symbolic_omp(A, B) if parallel else symbolic(A, B)
     nnz = int(c_rpt[-1])
     c_col = np.empty(nnz, dtype=np.int32)
     c_val = np.empty(nnz, dtype=dtype)
-    c_abs = np.empty(nnz, dtype=np.float64)
-    fn = _lib().oracle_numeric_f64 if dtype == np.float64 else _lib().oracle_numeric_f32
+    c_abs = np.empty(nnz, dtype=np.float64) if (with_abs or not parallel) else None
+    if parallel:
+        fn = _lib().oracle_numeric_omp_f64 if dtype == np.float64 else _lib().oracle_numeric_omp_f32
+    else:
+        fn = _lib().oracle_numeric_f64 if dtype == np.float64 else _lib().oracle_numeric_f32
     if dtype not in (np.float64, np.float32):
         raise TypeError(dtype)
     rc = fn(A.m, B.m, B.n, _p(a_rpt), _p(a_col), _p(a_val), _p(b_rpt), _p(b_col), _p(b_val),

@@ -134,3 +134,118 @@ bad_count:                                                                      
 
 ORACLE_NUMERIC(oracle_numeric_f64, double)
 ORACLE_NUMERIC(oracle_numeric_f32, float)
+
+/* ----------------------------------------------------------------------------------------
+ * Row-parallel variants: the same two passes for timing the oracle on
+ * all host cores and for full-size parity checks (R-MAT s22/s23).  Rows of C are independent
+ * (Algorithm 1's outer loop), so each thread runs, for its rows, exactly the loops
+ * of oracle_symbolic / Algorithm 1 above on its own dense accumulator: every row is summed in
+ * Algorithm 1's product order, and the output is identical to the single-thread functions
+ * (tests/test_oracle_pins.py checks that bit for bit).  Compiled with -fopenmp when available;
+ * without it they run on one thread.  c_abs may be NULL (no tolerance scale).
+ * ---------------------------------------------------------------------------------------- */
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+int oracle_threads(void)
+{
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+
+/* pass 1: distinct columns per row -> c_rpt (exclusive prefix sums) */
+int oracle_symbolic_omp(int64_t m, int64_t k, int64_t n,
+                        const int64_t *a_rpt, const int32_t *a_col,
+                        const int64_t *b_rpt, const int32_t *b_col, int64_t *c_rpt)
+{
+    int err = 0;
+    c_rpt[0] = 0;
+#pragma omp parallel
+    {
+        int64_t *mark = (int64_t *)malloc((size_t)(n > 0 ? n : 1) * sizeof(int64_t));
+        if (!mark) {
+#pragma omp atomic write
+            err = -2;
+        } else {
+            for (int64_t j = 0; j < n; ++j) mark[j] = -1;
+#pragma omp for schedule(dynamic, 256)
+            for (int64_t i = 0; i < m; ++i) {
+                int64_t cnt = 0;
+                for (int64_t p = a_rpt[i]; p < a_rpt[i + 1]; ++p) {
+                    int32_t kk = a_col[p];
+                    if (kk < 0 || kk >= k) { err = -1; break; }
+                    for (int64_t q = b_rpt[kk]; q < b_rpt[kk + 1]; ++q) {
+                        int32_t j = b_col[q];
+                        if (j < 0 || j >= n) { err = -1; break; }
+                        if (mark[j] != i) { mark[j] = i; ++cnt; }
+                    }
+                }
+                c_rpt[i + 1] = cnt;  /* per-row count; scanned below */
+            }
+            free(mark);
+        }
+    }
+    if (err) return err;
+    for (int64_t i = 0; i < m; ++i) c_rpt[i + 1] += c_rpt[i];
+    return 0;
+}
+
+#define ORACLE_NUMERIC_OMP(NAME, VT)                                                    \
+int NAME(int64_t m, int64_t k, int64_t n,                                               \
+         const int64_t *a_rpt, const int32_t *a_col, const VT *a_val,                   \
+         const int64_t *b_rpt, const int32_t *b_col, const VT *b_val,                   \
+         const int64_t *c_rpt, int32_t *c_col, VT *c_val, double *c_abs)                \
+{                                                                                       \
+    int err = 0;                                                                        \
+    _Pragma("omp parallel")                                                             \
+    {                                                                                   \
+        int64_t *mark = (int64_t *)malloc((size_t)(n > 0 ? n : 1) * sizeof(int64_t));   \
+        VT *acc = (VT *)malloc((size_t)(n > 0 ? n : 1) * sizeof(VT));                   \
+        double *aacc = c_abs ? (double *)malloc((size_t)(n > 0 ? n : 1) * sizeof(double)) \
+                             : NULL;                                                    \
+        if (!mark || !acc || (c_abs && !aacc)) {                                        \
+            err = -2;                                                                   \
+        } else {                                                                        \
+            for (int64_t j = 0; j < n; ++j) mark[j] = -1;                               \
+            _Pragma("omp for schedule(dynamic, 256)")                                   \
+            for (int64_t i = 0; i < m; ++i) {                                           \
+                int32_t *list = c_col + c_rpt[i];                                       \
+                int64_t cnt = 0, cap = c_rpt[i + 1] - c_rpt[i];                          \
+                for (int64_t p = a_rpt[i]; p < a_rpt[i + 1] && !err; ++p) {             \
+                    int32_t kk = a_col[p];                                              \
+                    VT a = a_val[p];                                                    \
+                    if (kk < 0 || kk >= k) { err = -1; break; }                         \
+                    for (int64_t q = b_rpt[kk]; q < b_rpt[kk + 1]; ++q) {               \
+                        int32_t j = b_col[q];                                           \
+                        VT value = a * b_val[q];                /* value <- a_ik b_kj */ \
+                        if (j < 0 || j >= n) { err = -1; break; }                       \
+                        if (mark[j] != i) {                     /* absent: insert */    \
+                            if (cnt >= cap) { err = -3; break; }                        \
+                            mark[j] = i; acc[j] = value; list[cnt++] = j;               \
+                            if (aacc) aacc[j] = fabs((double)a) * fabs((double)b_val[q]); \
+                        } else {                                /* present: accumulate */ \
+                            acc[j] = acc[j] + value;                                    \
+                            if (aacc) aacc[j] += fabs((double)a) * fabs((double)b_val[q]); \
+                        }                                                               \
+                    }                                                                   \
+                }                                                                       \
+                if (err) continue;                                                      \
+                if (cnt != cap) { err = -3; continue; }                                 \
+                qsort(list, (size_t)cnt, sizeof(int32_t), cmp_i32);                     \
+                for (int64_t e = 0; e < cnt; ++e) {                                     \
+                    c_val[c_rpt[i] + e] = acc[list[e]];                                 \
+                    if (aacc) c_abs[c_rpt[i] + e] = aacc[list[e]];                      \
+                }                                                                       \
+            }                                                                           \
+        }                                                                               \
+        free(mark); free(acc); free(aacc);                                              \
+    }                                                                                   \
+    return err;                                                                         \
+}
+
+ORACLE_NUMERIC_OMP(oracle_numeric_omp_f64, double)
+ORACLE_NUMERIC_OMP(oracle_numeric_omp_f32, float)

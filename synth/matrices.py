@@ -5,7 +5,8 @@ intermediate-product counts, no binning.  It only builds matrix *structure* and
 *values* with the shapes of the paper's workloads (Table II),
 following the recipes of SURVEY.md §8(d) restated in DESIGN.md "Input recipe".
 
-All generators use NumPy PCG64 (`np.random.default_rng(seed)`) and return a `Csr`
+All generators use NumPy PCG64 (`np.random.default_rng(seed)`) except R-MAT (synth/rmat.c,
+a counter-based splitmix64 draw, compiled on first use) and return a `Csr`
 with int64 row pointers, int32 column indices (sorted, de-duplicated unless a
 generator says otherwise) and float64 values (callers cast to float32 for SP runs;
 both sides then see the identical rounded values).
@@ -218,27 +219,72 @@ def epidemiology_like(n: int = 725) -> Csr:
     return from_coo(n * n, n * n, np.concatenate(R), np.concatenate(C), name="epidemiology_like")
 
 
+_RMAT_SO = None
+
+
+def _rmat_lib():
+    """Compile synth/rmat.c (gcc -O3 -fopenmp) on first use and load it (ctypes)."""
+    global _RMAT_SO
+    if _RMAT_SO is None:
+        import ctypes
+        import os
+        import subprocess
+        here = os.path.dirname(os.path.abspath(__file__))
+        src, so = os.path.join(here, "rmat.c"), os.path.join(here, "librmat.so")
+        if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+            subprocess.check_call(["gcc", "-O3", "-fopenmp", "-shared", "-fPIC", "-o", so, src])
+        lib = ctypes.CDLL(so)
+        lib.rmat_csr.restype = ctypes.c_int64
+        lib.rmat_csr.argtypes = [ctypes.c_int, ctypes.c_int64, ctypes.c_double, ctypes.c_double, ctypes.c_double,
+                                 ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p]
+        _RMAT_SO = lib
+    return _RMAT_SO
+
+
 def rmat(scale: int, edge_factor: int = 16, a: float = 0.45, b: float = 0.15, c: float = 0.15,
-         seed: int = 1, chunk: int = 1 << 23) -> Csr:
-    """Config 5: R-MAT (a,b,c,d) directed graph, duplicates merged, no relabelling."""
-    rng = np.random.default_rng(seed)
+         seed: int = 1) -> Csr:
+    """Config 5: R-MAT (a,b,c,d) directed graph, duplicates merged, no relabelling
+    (synth/rmat.c: counter-based draws, OpenMP; s22 in ~1 s on 8 cores)."""
+    N = 1 << scale
+    rpt = np.empty(N + 1, dtype=np.int64)
+    col = np.empty(edge_factor * N, dtype=np.int32)
+    nnz = _rmat_lib().rmat_csr(scale, edge_factor, a, b, c, seed, rpt.ctypes.data, col.ctypes.data)
+    if nnz < 0:
+        raise MemoryError("rmat_csr: out of host memory")
+    return Csr(N, N, rpt, col[:nnz].copy(), None, f"rmat{scale}")
+
+
+_M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
+
+
+def _mix64(z: np.ndarray) -> np.ndarray:
+    """splitmix64 finaliser on uint64 arrays (wrapping arithmetic), as in synth/rmat.c."""
+    z = z + np.uint64(0x9E3779B97F4A7C15)
+    z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+    z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+    return z ^ (z >> np.uint64(31))
+
+
+def _rmat_numpy(scale: int, edge_factor: int = 16, a: float = 0.45, b: float = 0.15, c: float = 0.15,
+                seed: int = 1) -> Csr:
+    """The same generator as synth/rmat.c in NumPy (small scales; cross-check of the C build)."""
     N = 1 << scale
     E = edge_factor * N
-    keys = []
-    for s in range(0, E, chunk):
-        e = min(E, s + chunk)
-        r = np.zeros(e - s, dtype=np.int64)
-        q = np.zeros(e - s, dtype=np.int64)
-        for lvl in range(scale):
-            u = rng.random(e - s)
-            r |= (u >= a + b).astype(np.int64) << lvl
-            q |= (((u >= a) & (u < a + b)) | (u >= a + b + c)).astype(np.int64) << lvl
-        keys.append(np.unique(r * N + q))
-    key = np.unique(np.concatenate(keys))
-    r = key // N
-    col = (key - r * N).astype(np.int32)
+    s0 = _mix64(np.array([seed], dtype=np.uint64))[0]
+    e = np.arange(E, dtype=np.uint64)
+    r = np.zeros(E, dtype=np.int64)
+    q = np.zeros(E, dtype=np.int64)
+    ab, abc = a + b, a + b + c
+    for lvl in range(scale):
+        x = _mix64(s0 ^ (e * np.uint64(64) + np.uint64(lvl)))
+        u = (x >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+        r |= (u >= ab).astype(np.int64) << lvl
+        q |= (((u >= a) & (u < ab)) | (u >= abc)).astype(np.int64) << lvl
+    key = np.unique(r * N + q)
+    rr = key // N
+    col = (key - rr * N).astype(np.int32)
     rpt = np.zeros(N + 1, dtype=np.int64)
-    np.cumsum(np.bincount(r, minlength=N), out=rpt[1:])
+    np.cumsum(np.bincount(rr, minlength=N), out=rpt[1:])
     return Csr(N, N, rpt, col, None, f"rmat{scale}")
 
 

@@ -322,3 +322,46 @@ def test_bin_of_table1_p100():
     keys = np.random.default_rng(0).integers(0, 20000, size=10000)
     h = oracle.binning.group_histogram(keys, [32, 512, 1024, 2048, 4096, 8192])
     assert h.sum() == (keys > 0).sum()
+
+
+# ----------------------------------------------------------------- working precision (R10)
+
+@pytest.mark.parametrize("parallel", [False, True])
+def test_fp32_working_precision(parallel):
+    """Reading R10 (value tables of 4 B for SP): products and sums are rounded to
+    fp32 in Algorithm 1's order.  Row 0: products 2^24, 1, -2^24 (in that order) sum to 0 in fp32
+    (2^24 + 1 rounds to 2^24, ties-to-even) and to 1 in fp64.  Row 1: one product
+    (1 + 2^-12)^2 = 1 + 2^-11 + 2^-24 rounds to 1 + 2^-11 in fp32 (tie, even mantissa) and is
+    exact in fp64.  An oracle accumulating or multiplying in double fails the fp32 half."""
+    x = 1.0 + 2.0 ** -12
+    # A row 0 = [1, 1, 1] at cols 0..2, row 1 = [x] at col 0; B rows 0..2 = 2^24, 1, -2^24 at col 0
+    B = Csr(3, 1, np.array([0, 1, 2, 3], dtype=np.int64), np.array([0, 0, 0], dtype=np.int32),
+            np.array([2.0 ** 24, 1.0, -2.0 ** 24]))
+    A2 = Csr(2, 3, np.array([0, 3, 4], dtype=np.int64), np.array([0, 1, 2, 0], dtype=np.int32),
+             np.array([1.0, 1.0, 1.0, x]))
+    rpt, col, v32, _ = oracle.spgemm(A2.astype(np.float32), B.astype(np.float32), np.float32, parallel=parallel)
+    assert rpt.tolist() == [0, 1, 2] and col.tolist() == [0, 0]
+    assert v32[0] == np.float32(0.0)
+    assert v32[1] == np.float32(x * 2.0 ** 24)  # row 1 = x * b_00 = x * 2^24: exact in fp32
+    rpt, col, v64, _ = oracle.spgemm(A2, B, np.float64, parallel=parallel)
+    assert v64[0] == 1.0
+    # the product rounding itself: (1 + 2^-12) * (1 + 2^-12) with both factors fp32
+    P = Csr(1, 1, np.array([0, 1], dtype=np.int64), np.array([0], dtype=np.int32), np.array([x]))
+    _, _, p32, _ = oracle.spgemm(P.astype(np.float32), P.astype(np.float32), np.float32, parallel=parallel)
+    _, _, p64, _ = oracle.spgemm(P, P, np.float64, parallel=parallel)
+    assert p32[0] == np.float32(1.0 + 2.0 ** -11)
+    assert p64[0] == 1.0 + 2.0 ** -11 + 2.0 ** -24
+
+
+@pytest.mark.parametrize("name,dtype", [("rmat12", np.float32), ("mixed:economics", np.float64),
+                                        ("poisson64", np.float64)])
+def test_parallel_oracle_identical(name, dtype):
+    """the row-parallel oracle equals the single-thread one bit for bit
+    (every row is still summed in Algorithm 1 order)."""
+    A = synth.config(name).astype(dtype)
+    s = oracle.spgemm(A, A, dtype)
+    p = oracle.spgemm(A, A, dtype, parallel=True)
+    for x, y in zip(s, p):
+        assert np.array_equal(x, y)
+    assert np.array_equal(oracle.symbolic_omp(A, A), s[0])
+    assert oracle.threads() >= 1 and oracle.cores() >= 1

@@ -79,3 +79,11 @@ def test_values_recipes():
     v = synth.values(10000, "uniform", 1)
     assert v.min() >= -1 and v.max() <= 1
     assert np.array_equal(synth.values(100, "uniform", 3), synth.values(100, "uniform", 3))
+
+
+@pytest.mark.parametrize("scale,seed", [(6, 1), (10, 1), (12, 5)])
+def test_rmat_c_matches_numpy_twin(scale, seed):
+    """synth/rmat.c (OpenMP, counter-based draws) equals its NumPy twin exactly."""
+    from synth.matrices import _rmat_numpy
+    A, B = synth.rmat(scale, seed=seed), _rmat_numpy(scale, seed=seed)
+    assert np.array_equal(A.rpt, B.rpt) and np.array_equal(A.col, B.col)
