@@ -177,13 +177,26 @@ typedef enum {
                                        keep the paper hash on their small-row groups (the level-1
                                        clear + prefix costs more than the row).  Default 500,
                                        0 = no limit */
-    SPGEMM_OPT_RANK_L1_PCT_SYM = 20 /* same for the symbolic rank-count kernels, B = the group's
+    SPGEMM_OPT_RANK_L1_PCT_SYM = 20,/* same for the symbolic rank-count kernels, B = the group's
                                        n_prod bound.  Default 150, 0 = no limit */
+    SPGEMM_OPT_BATCH = 21,          /* batched graph-row kernels, bit mask:
+                                       1 = symbolic groups 2-9 by the paper hash (Alg. 5), R rows
+                                       of one group per CTA with their products flattened;
+                                       2 = numeric expand-bucket-rank (ESC) for rows of symbolic
+                                       groups 2-8 with 100 * n_prod_i <= ESC_PCT * nnz_i (needs
+                                       RANGE_HASH: column spans).  Default 2 (the batched symbolic
+                                       kernels measured slower than the per-group ones on R-MAT
+                                       s22); 0 = off (ablation).
+                                       Off while the matching MIN_GROUP is forced */
+    SPGEMM_OPT_ESC_PCT = 22,        /* compression bound of the ESC rows (default 200: n_prod_i <=
+                                       2 nnz_i) */
+    SPGEMM_OPT_ESC_GROUPS = 23      /* bit g: rows of symbolic group g (2..8) may take the ESC kernels;
+                                       -1 (default) = the library's rule */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);
 
-#define SPGEMM_MAX_GROUPS 16
+#define SPGEMM_MAX_GROUPS 24
 
 /* Counters of the last symbolic/numeric call.  Times are CUDA-event milliseconds measured on
  * the stream each kernel was launched on (group kernels: their own stream). */
@@ -215,7 +228,9 @@ typedef enum {
     SPGEMM_KERNEL_CLUSTER = 4,  /* distributed shared-memory hash table (kernels_cluster.cu)     */
     SPGEMM_KERNEL_GLOBAL = 5,   /* global-memory hash table                  */
     SPGEMM_KERNEL_RANK_BIG = 6, /* rank-indexed, level 2 in global memory, values reduced into C */
-    SPGEMM_KERNEL_TINY = 7      /* thread per row, sorted register table (kernels_tiny.cu)       */
+    SPGEMM_KERNEL_TINY = 7,     /* thread per row, sorted register table (kernels_tiny.cu)       */
+    SPGEMM_KERNEL_BATCH = 8,    /* batched rows per CTA, paper hash in shared memory (symbolic)   */
+    SPGEMM_KERNEL_ESC = 9       /* batched expand-bucket-rank-compress rows (kernels_esc.cu)      */
 } spgemm_kernel_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);
@@ -223,7 +238,7 @@ SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *o
 /* Group table of the implementation: inclusive upper bounds of each group's key (n_prod
  * for phase 1, nnz for phase 2), ascending; the group after the last bound is the global-
  * memory fallback.  *ngroups (host) receives the number of bounds. */
-SPGEMM_API spgemm_status_t spgemm_group_bounds(int phase /* 1 or 2 */, int64_t *upper /* host, >= 16 */,
+SPGEMM_API spgemm_status_t spgemm_group_bounds(int phase /* 1 or 2 */, int64_t *upper /* host, >= 24 */,
                                     int32_t *ngroups /* host */);
 
 /* Copy the per-row n_prod (int64, m) and the grouping permutation of `phase` (int32, m:

@@ -317,12 +317,14 @@ cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int3
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows) {
   if (max_rows <= 0) return cudaSuccess;
   constexpr int smem = kClusterSymSlots * 4;
-  static int nc = 0;
-  if (nc == 0) {
+  static PerDevice ncache;
+  auto& ncd = ncache.here();
+  if (ncd.load() == 0) {
     cudaError_t e = set_cluster_attrs(k_sym_cluster<kClusterSize>, smem);
     if (e != cudaSuccess) return e;
-    nc = max_clusters(k_sym_cluster<kClusterSize>, kClusterSize, smem);
+    ncd.store(max_clusters(k_sym_cluster<kClusterSize>, kClusterSize, smem));
   }
+  const int nc = (int)ncd.load();
   SymArgs b = a;
   if (b.vw_log2 > 5) b.vw_log2 = 5;
   const int grid = max_rows < nc ? max_rows : nc;
@@ -333,12 +335,14 @@ cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int3
 template <typename VT, int CS>
 cudaError_t launch_num_cluster_cs(cudaStream_t s, const NumArgs& a, int* nclusters_out) {
   constexpr int smem = kClusterNumSlots * ((int)sizeof(VT) + 4);
-  static int nc = 0;
-  if (nc == 0) {
+  static PerDevice ncache;
+  auto& ncd = ncache.here();
+  if (ncd.load() == 0) {
     cudaError_t e = set_cluster_attrs(k_num_cluster<VT, CS>, smem);
     if (e != cudaSuccess) return e;
-    nc = max_clusters(k_num_cluster<VT, CS>, CS, smem);
+    ncd.store(max_clusters(k_num_cluster<VT, CS>, CS, smem));
   }
+  const int nc = (int)ncd.load();
   if (nclusters_out) { *nclusters_out = nc; return cudaSuccess; }  // query only
   if (a.nrows <= 0) return cudaSuccess;
   NumArgs b = a;

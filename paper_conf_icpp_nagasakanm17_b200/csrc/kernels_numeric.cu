@@ -638,12 +638,13 @@ __global__ __launch_bounds__(1024) void k_num_global(NumArgs a) {
 
 template <typename VT, int T, int TPR, int BS, long long UPPER, bool RANK2>
 cudaError_t launch_num_k(cudaStream_t s, const NumArgs& a, int smem) {
-  static int configured = 0;
-  if (smem > configured) {
+  static PerDevice configured;
+  auto& cfg = configured.here();
+  if (smem > cfg.load()) {
     cudaError_t e = cudaFuncSetAttribute(k_num_smem<VT, T, TPR, BS, UPPER, RANK2>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    configured = smem;
+    cfg.store(smem);
   }
   NumArgs b = a;
   const int max_vw = TPR < 32 ? TPR : 32;

@@ -511,10 +511,11 @@ int range_grid(K kernel, int threads, size_t smem, int num_sms, long long nrows,
 }
 
 template <typename K>
-cudaError_t set_smem(K kernel, size_t smem, size_t& configured) {
-  if (smem <= configured) return cudaSuccess;
+cudaError_t set_smem(K kernel, size_t smem, PerDevice& cache) {
+  auto& configured = cache.here();
+  if ((long long)smem <= configured.load()) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess) configured = smem;
+  if (e == cudaSuccess) configured.store((long long)smem);
   return e;
 }
 
@@ -544,7 +545,7 @@ cudaError_t launch_symbolic_range(cudaStream_t s, const SymArgs& a, int rmax, in
   const long long per = (long long)sizeof(RMetaW<int>) + rcap;
   const int warps = range_warps(per);
   const size_t smem = (size_t)warps * per;
-  static size_t configured = 0;
+  static PerDevice configured;
   cudaError_t e = set_smem(k_sym_range, smem, configured);
   if (e != cudaSuccess) return e;
   const int grid = range_grid(k_sym_range, warps * 32, smem, num_sms, a.nrows, warps);
@@ -577,7 +578,7 @@ static cudaError_t launch_num_range_t(cudaStream_t s, const NumArgs& a, int rcap
   const long long per = (long long)sizeof(RMetaW<VT>) + (long long)NC * rcap * sizeof(VT);
   const int warps = range_warps(per, range_num_budget<VT>());
   const size_t smem = (size_t)warps * per;
-  static size_t configured = 0;
+  static PerDevice configured;
   cudaError_t e = set_smem(k_num_range<VT, NC>, smem, configured);
   if (e != cudaSuccess) return e;
   const int grid = range_grid(k_num_range<VT, NC>, warps * 32, smem, num_sms, a.nrows, warps);

@@ -346,14 +346,15 @@ __global__ __launch_bounds__(TPR, rank_min_blocks<TPR, 4>()) void k_sym_rankcnt(
 }
 
 template <typename K>
-cudaError_t prepare(K kernel, int smem, int& configured) {
-  if (smem > configured) {
+cudaError_t prepare(K kernel, int smem, PerDevice& cache) {
+  auto& configured = cache.here();
+  if (smem > configured.load()) {
     cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     // the rows' B gathers are scattered (L1 hit rates ~30%): give the SM's memory to the tables
     e = cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
-    configured = smem;
+    configured.store(smem);
   }
   return cudaSuccess;
 }
@@ -364,7 +365,7 @@ cudaError_t launch_rankacc_k(cudaStream_t s, const NumArgs& a) {
   constexpr long long UPPER = kNumGroups[G].upper;
   using L = RankLayout<VT, true, c.TPR, UPPER, c.MC, c.KP>;
   const int smem = L::bytes(a.l1_words);
-  static int configured = 0;
+  static PerDevice configured;
   cudaError_t e = prepare(k_num_rankacc<VT, c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
   k_num_rankacc<VT, c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
@@ -377,7 +378,7 @@ cudaError_t launch_rankcnt_k(cudaStream_t s, const SymArgs& a) {
   constexpr long long UPPER = kSymGroups[G].upper;
   using L = RankLayout<int, false, c.TPR, UPPER, c.MC, c.KP>;
   const int smem = L::bytes(a.l1_words);
-  static int configured = 0;
+  static PerDevice configured;
   cudaError_t e = prepare(k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
   k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
@@ -504,7 +505,7 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
 template <typename VT>
 cudaError_t launch_rankbig_v(cudaStream_t s, const NumArgs& a, int grid) {
   const int smem = rankbig_smem_bytes_v<VT>(a.l1_words);
-  static int configured = 0;
+  static PerDevice configured;
   cudaError_t e = prepare(k_num_rankbig<VT>, smem, configured);
   if (e != cudaSuccess) return e;
   k_num_rankbig<VT><<<grid, 1024, smem, s>>>(a);

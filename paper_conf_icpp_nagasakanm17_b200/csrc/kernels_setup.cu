@@ -388,7 +388,7 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(long long m, cons
                                                                long long* __restrict__ tile_sums,
                                                                const uint8_t* __restrict__ grp1,
                                                                uint8_t* __restrict__ grp2, DevAcc* __restrict__ acc,
-                                                               Bounds bd) {
+                                                               Bounds bd, EscSel esc) {
   __shared__ long long ws[33];
   __shared__ int s_cnt[kMaxGroups];
   __shared__ unsigned long long s_max;
@@ -409,7 +409,14 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_reduce(long long m, cons
     if (grouping) {  // block-uniform branch
       int g = -1;
       if (i < m) {
-        if (v > 0) g = (bd.range_group >= 0 && grp1[i] == kSymRange) ? bd.range_group : group_of(v, bd);
+        if (v > 0) {
+          const int g1 = grp1[i];
+          if (bd.range_group >= 0 && g1 == kSymRange) g = bd.range_group;
+          else if (esc.nprod && g1 >= kEscSymLo && g1 <= kEscSymHi && ((esc.groups >> g1) & 1u) &&
+                   100 * esc.nprod[i] <= (long long)esc.pct * v)
+            g = kNumEscBase + g1 - kEscSymLo;
+          else g = group_of(v, bd);
+        }
         grp2[i] = (uint8_t)(g < 0 ? 0xFF : g);
       }
       count_group(g >= 0, g, s_cnt);
@@ -611,10 +618,11 @@ size_t scan_workspace_bytes(long long m) {
 }
 
 static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const uint8_t* grp1, uint8_t* grp2,
-                                  DevAcc* acc, Bounds b, long long* tile_ws, long long* total_out, int* nlaunch) {
+                                  DevAcc* acc, Bounds b, EscSel esc, long long* tile_ws, long long* total_out,
+                                  int* nlaunch) {
   if (m == 0) return cudaSuccess;
   const long long ntiles = (m + kScanTile - 1) / kScanTile;
-  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, grp1, grp2, acc, b);
+  k_scan_reduce<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, grp1, grp2, acc, b, esc);
   k_scan_tiles<<<1, 1024, 0, s>>>(ntiles, tile_ws);
   k_scan_down<<<(unsigned)ntiles, kSetupThreads, 0, s>>>(m, x, tile_ws, total_out);
   if (nlaunch) *nlaunch += 3;
@@ -622,8 +630,9 @@ static cudaError_t scan_inclusive(cudaStream_t s, long long m, int64_t* x, const
 }
 
 cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const uint8_t* grp1,
-                                  uint8_t* grp2, DevAcc* acc, Bounds b, long long* tile_ws, int* nlaunch) {
-  return scan_inclusive(s, m, c_rpt + 1, grp1, grp2, acc, b, tile_ws, &acc->nnzc, nlaunch);
+                                  uint8_t* grp2, DevAcc* acc, Bounds b, EscSel esc, long long* tile_ws,
+                                  int* nlaunch) {
+  return scan_inclusive(s, m, c_rpt + 1, grp1, grp2, acc, b, esc, tile_ws, &acc->nnzc, nlaunch);
 }
 
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
@@ -642,7 +651,8 @@ cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, 
     k_nprod_only<<<(unsigned)((m + rpb - 1) / rpb), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, nprod_scan + 1);
     Bounds none{};
     none.range_group = -1;
-    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, nullptr, none, tile_ws, nullptr, nlaunch);
+    e = scan_inclusive(s, m, nprod_scan + 1, nullptr, nullptr, nullptr, none, EscSel{nullptr, 0, 0u}, tile_ws, nullptr,
+                       nlaunch);
     if (e != cudaSuccess) return e;
   }
   k_splits<<<(nparts + 1 + 255) / 256, 256, 0, s>>>(m, nprod_scan, nparts, splits_dev);

@@ -194,12 +194,13 @@ cudaError_t launch_sym(cudaStream_t s, const SymArgs& a) {
   constexpr int RPB = BS / TPR;
   constexpr int smem = RPB * T * 4;
   static_assert(smem <= kSmemLimit - 1024, "symbolic table too large");
-  static bool configured = false;
-  if (!configured) {
+  static PerDevice configured;
+  auto& cfg = configured.here();
+  if (!cfg.load()) {
     cudaError_t e = cudaFuncSetAttribute(k_sym_smem<T, TPR, BS, OPT>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    configured = true;
+    cfg.store(1);
   }
   SymArgs b = a;
   const int max_vw = TPR < 32 ? TPR : 32;

@@ -95,6 +95,12 @@ struct spgemm_ctx {
   // vs 4.5, group 7 (4096) 3.6 vs 4.6
   long long rank_l1_pct = 500, rank_l1_pct_sym = 150;
   int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
+  // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
+  // 26.5 ms vs 21.7 ms with the per-group hash / rank-count kernels), bit 2 numeric ESC
+  int batch = 2;
+  long long esc_pct = 200;  // numeric ESC rows: 100 * n_prod_i <= esc_pct * nnz_i
+  long long esc_mask = -1;  // symbolic groups whose rows may take the numeric ESC kernels (-1: auto)
+  long long esc_w_pct = 200;  // auto rule: ESC where 100 * (n/1024 + 1) >= esc_w_pct * group bound
   bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)
   // CTA-per-row numeric hash groups: two-level bitmap rank (else bucket sort); 1 = only where the
   // level-1 width W <= the group's nnz bound (R-MAT s22, W = 4097: bucket 4.1 ms vs bitmap 21.9 ms
@@ -361,6 +367,23 @@ bool flat_of(spgemm_handle_t h) {
   return h->k > 0 && (double)h->nnzb / (double)h->k < 16.0;
 }
 
+// Symbolic groups whose weakly compressing rows take the numeric ESC kernels (kernels_esc.cu)
+// instead of the rank-indexed CTA-per-row kernels, whose level-1 bitmap costs W = n/1024 + 1 words
+// per row whatever the row's size: ESC where 100 * W >= esc_w_pct * B (B = the group's n_prod
+// bound).  Measured per group (scripts/esc_groups.py, serial, fp32): R-MAT s22 (W = 4097) ESC
+// saves 1.7 / 1.3 / 3.4 / 5.8 / 2.0 ms on groups 2-6 (W/B = 32 .. 2) and loses 1.8 / 1.9 ms on
+// groups 7-8 (W/B = 1, 0.5); R-MAT s20 (W = 1025) saves 0.4 / 0.1 ms on groups 2-3 (W/B = 8, 4),
+// loses 0.2 ms on group 4 (W/B = 2); webbase, R-MAT s16/s18, Economics, Circuit lose on every
+// group (W <= 1024: their level-1 bitmaps are cheap; webbase's 95 %-local rows also skew the
+// buckets, which costs the ESC kernels a refinement pass).
+unsigned esc_auto_mask(spgemm_handle_t h) {
+  const long long W = h->n / 1024 + 1;
+  unsigned m = 0;
+  for (int g = kEscSymLo; g <= kEscSymHi; ++g)
+    if (100 * W >= h->esc_w_pct * kSymGroups[g].upper && W > 1024) m |= 1u << g;
+  return m;
+}
+
 int long_len_of(spgemm_handle_t h) {
   if (h->long_len < 0) return 0;
   if (h->long_len > 0) return h->long_len;
@@ -549,6 +572,13 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_TINY:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "TINY must be 0, 1 or 2");
       h->tiny = (int)v; break;
+    case SPGEMM_OPT_BATCH:
+      if (v < 0 || v > 3) return fail(h, SPGEMM_ERR_INVALID_ARG, "BATCH must be 0..3");
+      h->batch = (int)v; break;
+    case SPGEMM_OPT_ESC_PCT:
+      if (v < 0 || v > (1LL << 40)) return fail(h, SPGEMM_ERR_INVALID_ARG, "ESC_PCT out of range");
+      h->esc_pct = v; break;
+    case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -607,8 +637,14 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   }
   if (h->timing) CK(cudaEventRecord(h->ev[0], h->stream));
   if (h->validate) {
+    // checked before any kernel indexes B through col_A or walks rpt (an out-of-range column
+    // would otherwise fault in the n_prod pass instead of returning SPGEMM_ERR_INVALID_INPUT)
     CK(launch_validate(h->stream, m, k, n, a_rpt, a_col, b_rpt, b_col, &dacc->err_flags));
     ++launches;
+    CK(cudaMemcpyAsync(&h->hacc->err_flags, &dacc->err_flags, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    CK(cudaStreamSynchronize(h->stream));
+    if (h->hacc->err_flags & 1)
+      return fail(h, SPGEMM_ERR_INVALID_INPUT, "input validation failed (rpt not monotone or col out of range)");
   }
   // (1)+(2): n_prod per row (Alg. 2), column spans, group ids / histogram
   {
@@ -671,6 +707,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.n = n;
   sa.l1_words = (int)((n + 1023) / 1024 + 1);
   sa.err_flags = &dacc->err_flags;
+  // batched paper-hash symbolic kernels for groups 2-9 (kernels_esc.cu)
+  auto batch_sym_on = [&](int g) { return (h->batch & 1) && h->sym_min_group < 0 && g >= 2 && g <= 9; };
   // rank-count kernels for the CTA-per-row groups (kernels_rankacc.cu; needs the column spans)
   auto rank_cnt_on = [&](int g) {
     return h->rank_acc && h->rlohi.p != nullptr && h->sym_min_group < 0 && g >= 5 && g <= 9 &&
@@ -705,7 +743,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->use_cluster, h->cluster_fill, h->use_streams, h->timing, h->num_min_group,
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
-                                 (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym};
+                                 (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym,
+                                 (long long)h->sym_min_group, (long long)h->batch, h->esc_pct, h->esc_mask};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -734,9 +773,11 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       ga.nrows = rows;
       const bool tiny_g = h->tiny >= 2 && h->sym_min_group < 0 && g <= 1;  // measured slower than the hash
       if (tiny_g) CK(launch_symbolic_tiny(s, g, ga));
+      else if (batch_sym_on(g)) CK(launch_symbolic_batch(s, g, ga));
       else if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
       else CK(launch_symbolic_group(s, g, ga, h->num_sms));
-      h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
+      h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : batch_sym_on(g) ? SPGEMM_KERNEL_BATCH
+                     : rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
       ++launches;
       if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
         SymArgs gb = sa;
@@ -801,8 +842,12 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
 
     // (4) rpt_C = prefix sum, fused with (6) grouping by nnz_i
     int nl = 0;
+    // batched numeric rows need the column spans (bucket ranges) and no forced numeric group
+    const bool esc_on = (h->batch & 2) && h->rlohi.p != nullptr && h->num_min_group < 0;
+    const EscSel esc{esc_on ? static_cast<const int64_t*>(h->nprod.p) : nullptr, (int)std::min<long long>(h->esc_pct, 1 << 30),
+                     (unsigned)(h->esc_mask < 0 ? esc_auto_mask(h) : h->esc_mask)};
     CK(launch_scan_and_group(h->stream, m, c_rpt, static_cast<const uint8_t*>(h->grp1.p),
-                             static_cast<uint8_t*>(h->grp2.p), dacc, num_bounds(h),
+                             static_cast<uint8_t*>(h->grp2.p), dacc, num_bounds(h), esc,
                              static_cast<long long*>(h->tiles.p), &nl));
     launches += nl;
     
@@ -895,6 +940,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     na.priv_ok = h->snap1.b_unsorted ? 0 : 1;
     na.err_flags = &dacc->err_flags;
     na.l1_words = h->bitmap_rank ? (int)((h->n + 1023) / 1024 + 1) : 0;
+    na.nprod = static_cast<const int64_t*>(h->nprod.p);
     // rank-indexed accumulation for the CTA-per-row groups (needs the column spans; the forced
     // paths keep the paper hash)
     const int l1w_rank = (int)((h->n + 1023) / 1024 + 1);
@@ -952,7 +998,9 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     std::vector<long long> topo = {2, (long long)fp64, glob_grid, ctotal, btotal, h->vw_log2, na.long_len, na.flat,
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
-                                   (long long)low_compression, h->rank_l1_pct};
+                                   (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
+                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->snap2.max_nnz,
+                                   na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
@@ -972,7 +1020,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
         NumArgs ga = na;
         ga.rows = perm2 + off2.off[g];
         ga.nrows = rows;
-        if (g == kNumGlobal) {
+        if (g >= kNumEscBase) {  // batched expand-bucket-rank rows (kernels_esc.cu)
+          h->gkind[1][g] = SPGEMM_KERNEL_ESC;
+          CK(launch_numeric_esc(st, g - kNumEscBase + kEscSymLo, fp64, ga));
+        } else if (g == kNumGlobal) {
           h->gkind[1][g] = SPGEMM_KERNEL_GLOBAL;
           CK(launch_numeric_global(st, fp64, ga, glob_grid));
         } else if (g == kNumRange) {

@@ -14,12 +14,13 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <climits>
 
 namespace spg {
 
 constexpr unsigned kHashScal = 107u;  // HASH_SCAL; any odd constant (reading R4)
-constexpr int kMaxGroups = 16;
+constexpr int kMaxGroups = 24;
 constexpr int kSmemLimit = 232448;     // 227 KB opt-in per CTA on sm_100
 
 // ----------------------------------------------------------------------------- group tables
@@ -72,7 +73,12 @@ constexpr int kNumNumBounds = 13;
 constexpr int kNumCluster = 10;  // groups 10, 11, 12: clusters of 2, 4, 8 CTAs
 constexpr int kNumGlobal = 13;
 constexpr int kNumRange = 14;       // range rows (kernels_range.cu)
-constexpr int kNumNumGroups = 15;
+// Batched expand-bucket-rank rows (kernels_esc.cu): numeric groups 15..21 hold the rows of
+// symbolic groups 2..8 whose n_prod_i <= ESC_PCT/100 * nnz_i (weak compression); a batch of them
+// fits one CTA because the symbolic group bounds n_prod_i.
+constexpr int kNumEscBase = 15;
+constexpr int kEscSymLo = 2, kEscSymHi = 8;
+constexpr int kNumNumGroups = kNumEscBase + (kEscSymHi - kEscSymLo + 1);  // 22
 
 // Range rows (kernels_range.cu): column span R_i <= kRangeMaxSpan and
 // R_i <= kRangeSpanPerProd * n_prod_i, n_prod_i in [range_min_np, kRangeMaxNprod] (one warp
@@ -98,6 +104,20 @@ template <typename VT>
 __host__ __device__ constexpr long long num_cta_bytes(int T, long long upper, long long l1) {
   return align16(T * (int)sizeof(VT) + T * 4 + (int)upper * 6) + l1 * 8 + 16;
 }
+
+// ----------------------------------------------------------------------------- per-device setup
+// One-time per-kernel settings (dynamic shared memory opt-in, cluster occupancy) belong to the
+// device context, so launchers keep them per device ordinal; atomics make concurrent first
+// launches from several host threads safe (a setting applied twice is harmless).
+constexpr int kMaxDevices = 64;
+struct PerDevice {
+  std::atomic<long long> v[kMaxDevices] = {};
+  std::atomic<long long>& here() {
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess || d < 0) d = 0;
+    return v[d % kMaxDevices];
+  }
+};
 
 // ----------------------------------------------------------------------------- device state
 struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned host at the syncs
@@ -749,6 +769,7 @@ struct NumArgs {
   const unsigned* rbits; long long rwcap;  // range rows: symbolic pattern bitmap (same row order)
   int l1_words;            // CTA-per-row groups: level-1 words of the two-level rank (>= n/1024 + 1)
   unsigned long long* prof;  // diagnostics (SPGEMM_PROF_GROUP): per CTA row, %globaltimer at phase ends
+  const int64_t* nprod;      // batched kernels: n_prod_i of every row (step (1))
   int* row_counter;          // cluster groups: dynamic row counter (zeroed by spgemm_numeric)
 };
 
@@ -766,8 +787,15 @@ cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1,
                                const int64_t* nprod, const int64_t* a_rpt, const int64_t* c_rpt, DevAcc* acc);
 cudaError_t launch_group_scatter(cudaStream_t s, long long m, const uint8_t* grp, Offsets off,
                                  int* cursor, int32_t* perm);
+// Step-(6) selection of the batched numeric rows (kernels_esc.cu): rows of symbolic groups
+// kEscSymLo..kEscSymHi with 100 * n_prod_i <= pct * nnz_i go to group kNumEscBase + g1 - kEscSymLo.
+struct EscSel {
+  const int64_t* nprod;  // null: off
+  int pct;
+  unsigned groups;       // bit g: symbolic group g may take the ESC kernels
+};
 cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, const uint8_t* grp1,
-                                  uint8_t* grp2, DevAcc* acc, Bounds b,
+                                  uint8_t* grp2, DevAcc* acc, Bounds b, EscSel esc,
                                   long long* tile_ws, int* nlaunch);
 size_t scan_workspace_bytes(long long m);
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
@@ -801,6 +829,9 @@ int range_warps(long long per_warp, long long budget_default = kRangeSmemBudget)
 int range_rcap(long long rmax);
 int range_wcap(long long rmax);
 int cluster_capacity_sym();
+cudaError_t launch_symbolic_batch(cudaStream_t s, int group, const SymArgs& a);
+cudaError_t launch_numeric_esc(cudaStream_t s, int sym_group, bool fp64, const NumArgs& a);
+bool numeric_esc_supported(int sym_group, bool fp64);
 int cluster_capacity_num();
 
 }  // namespace spg

@@ -25,7 +25,7 @@ def main():
     starts = [i for i, (k, _) in enumerate(out) if "k_brow_minmax" in k or "k_nprod_group" in k]
     starts = [i for i in starts if i == 0 or "k_brow_minmax" not in out[i - 1][0]]
     step = out[starts[-1]:] if starts else out
-    lib = [(k, t) for k, t in step if "spg" in k]
+    lib = [(k, t) for k, t in step if "spg" in k or "k_" in k]
     tot = sum(t for _, t in lib)
     print(f"# ncu launch list — {title}\n")
     print("`ncu --metrics gpu__time_duration.sum --clock-control none`, one `bench.py` step with one stream "

@@ -58,7 +58,7 @@ def test_host_queries(lib):
         assert len(b) >= 7 and b == sorted(b) and len(set(b)) == len(b)
     assert lib.spgemm_status_string(0) == b"SPGEMM_OK"
     assert lib.spgemm_status_string(5) == b"SPGEMM_ERR_INDEX_OVERFLOW"
-    arr = (ctypes.c_int64 * 16)()
+    arr = (ctypes.c_int64 * 24)()
     n = ctypes.c_int32()
     assert lib.spgemm_group_bounds(3, arr, ctypes.byref(n)) == 1  # INVALID_ARG
     assert lib.spgemm_set_option(None, 0, 0) == 1

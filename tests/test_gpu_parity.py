@@ -674,3 +674,112 @@ def test_tiny_rows_int_exact_and_duplicates(spg):
         M.val[:] = M.val[o]
     got = check(spg, A, B, np.float32, exact=True, opts={"tiny": 2}, what="tiny dup int")
     assert got[3]["num_kernel"][0] == 7 and got[3]["sym_kernel"][0] == 7
+
+
+# ------------------------------------------------------------------ batched kernels (kernels_esc.cu)
+# Numeric ESC rows (expand, bucket, in-bucket rank, compress; one CTA per batch of rows of one
+# symbolic group) and the batched paper-hash symbolic kernels.  ESC_GROUPS forces every symbolic
+# group 2-8 onto ESC whatever the library's rule (which only picks them at R-MAT s22 scale).
+
+ESC_ALL = sum(1 << g for g in range(2, 9))
+
+
+def _esc_kernels(st):
+    return [g for g in range(15, 22) if st["num_rows"][g]]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("name", ["rmat14", "rmat16", "webbase_small", "mixed:circuit", "mixed:economics"])
+def test_esc_numeric(spg, name, dtype):
+    A = _mixed_small() if name == "webbase_small" else (
+        synth.rmat(int(name[4:])).with_values("uniform", 9) if name.startswith("rmat") else synth.config(name))
+    got = check(spg, A, A, dtype, opts={"esc_groups": ESC_ALL}, what=f"{name} esc")
+    st = got[3]
+    groups = _esc_kernels(st)
+    assert groups, "no rows took the ESC kernels"
+    assert all(st["num_kernel"][g] == 9 for g in groups), st["num_kernel"]
+
+
+@pytest.mark.parametrize("name", ["rmat14", "webbase_small"])
+def test_esc_int_exact(spg, name):
+    A = _mixed_small() if name == "webbase_small" else synth.rmat(14)
+    A = A.with_values("int", 3)
+    check(spg, A, A, np.float32, exact=True, opts={"esc_groups": ESC_ALL}, what=f"{name} esc int")
+
+
+def test_esc_duplicates_unsorted_and_compression(spg):
+    """Duplicate and unsorted columns inside A and B rows (equal keys: one entry, summed in the
+    run), and ESC_PCT large enough to send compressing rows through ESC as well."""
+    rng = np.random.default_rng(23)
+    m, n = 3000, 50000
+    rows = np.repeat(np.arange(m), 120)
+    cols = rng.integers(0, n, size=rows.size)
+    dup = rng.random(rows.size) < 0.3
+    cols[dup] = cols[np.maximum(np.arange(rows.size) - 1, 0)][dup]
+    A = from_coo(m, n, rows, cols, rng.uniform(-1, 1, rows.size), dedup=False)
+    B = from_coo(n, n, rng.integers(0, n, 400000), rng.integers(0, 12000, 400000),  # column band wider
+                 rng.uniform(-1, 1, 400000), dedup=False)                            # than range rows
+    for M in (A, B):
+        r = np.repeat(np.arange(M.m), np.diff(M.rpt))
+        o = np.lexsort((rng.random(r.size), r))
+        M.col[:] = M.col[o]
+        M.val[:] = M.val[o]
+    got = check(spg, A, B, np.float64, opts={"esc_groups": ESC_ALL, "esc_pct": 100000}, what="esc dup/unsorted")
+    assert _esc_kernels(got[3])
+
+
+@pytest.mark.parametrize("name", ["rmat16", "webbase_small", "mixed:qcd"])
+def test_batched_symbolic(spg, name):
+    """BATCH bit 1: symbolic groups 2-9 by the batched paper hash (Alg. 5 per row, rows of one
+    group flattened over a CTA)."""
+    A = _mixed_small() if name == "webbase_small" else (
+        synth.rmat(16).with_values("uniform", 5) if name == "rmat16" else synth.config(name))
+    got = check(spg, A, A, np.float32, opts={"batch": 3, "esc_groups": ESC_ALL}, what=f"{name} batched")
+    st = got[3]
+    assert any(st["sym_kernel"][g] == 8 for g in range(2, 10) if st["sym_rows"][g]), st["sym_kernel"]
+
+
+def test_esc_auto_rule_off_below_scale(spg):
+    """The library picks ESC only for wide matrices (n/1024 + 1 > 1024 level-1 words)."""
+    A = synth.rmat(16).with_values("uniform", 4)
+    got = check(spg, A, A, np.float32, what="rmat16 default")
+    assert not _esc_kernels(got[3])
+
+
+# ------------------------------------------------------------------ validation and graph keys
+
+def test_validate_rejects_bad_input(spg):
+    """SPGEMM_OPT_VALIDATE: an out-of-range column and a non-monotone rpt are reported as
+    SPGEMM_ERR_INVALID_INPUT before any kernel reads through them (and the handle stays usable)."""
+    A = synth.config("mixed:economics")
+    good = _dev(spg, A, np.float32)
+    with spg.Handle() as h:
+        h.set_option("validate", 1)
+        bad_col = spg.CsrMatrix(good.m, good.n, good.rpt.clone(), good.col.clone(), good.val)
+        bad_col.col[5] = good.n + 1000
+        with pytest.raises(spg.SpgemmError, match="INVALID_INPUT"):
+            h.multiply(bad_col, good)
+        bad_rpt = spg.CsrMatrix(good.m, good.n, good.rpt.clone(), good.col, good.val)
+        bad_rpt.rpt[10] = bad_rpt.rpt[12] + 1
+        with pytest.raises(spg.SpgemmError, match="INVALID_INPUT"):
+            h.multiply(bad_rpt, good)
+        torch.cuda.synchronize()
+        C = h.multiply(good, good)
+        ref = oracle.spgemm(A.astype(np.float32), A.astype(np.float32), np.float32)
+        assert_parity(C.numpy() + (None,), ref, np.float32, what="after rejected inputs")
+
+
+def test_graph_replay_new_structure_same_shape(spg):
+    """Two different structures with the same m, n, nnz(C)-independent pointers through one handle
+    (the numeric graph key includes max nnz_i and the global-table shape: ADVICE r1)."""
+    A1 = _mixed_small()
+    rng = np.random.default_rng(5)
+    A2 = synth.webbase_like(M=30000, seed=9, lmax=2500, alpha=1.5).with_values("uniform", 2)
+    with spg.Handle() as h:
+        for it, A in enumerate((A1, A2, A1, A2)):
+            h.set_option("num_min_group", 13 if it % 2 else -1)  # global group on odd calls
+            ref = oracle.spgemm(A.astype(np.float32), A.astype(np.float32), np.float32)
+            C = h.multiply(_dev(spg, A, np.float32), _dev(spg, A, np.float32))
+            torch.cuda.synchronize()
+            assert_parity(C.numpy() + (None,), ref, np.float32, what=f"call {it}")
+            del C
