@@ -1,22 +1,31 @@
-"""bench.py — SpGEMM GFLOPS (2*n_prod/s) of C = A^2 on B200.
+"""bench.py — SpGEMM GFLOPS (2*nprod/s) of C = A^2 on B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--config cant] [--dtype f32|f64]
+                    [--config rmat22] [--dtype f32|f64]
 
-One step = the whole hot path of SURVEY.md §8(a) on one synthetic input already resident in
-HBM: symbolic (n_prod, grouping, hash count, scan) -> exact allocation of C -> numeric
-(grouping, hash accumulate, gather, sort, write).  N=1 workload: BASELINE.json configs[1],
-the cant-like FEM matrix (62,451 rows, ~4.0M nnz), fp32.  N>1 (torchrun): weak scaling —
-rank p computes row block p of diag(A_0..A_{N-1})^2 with A_p a cant-like instance of seed p
-(the n_prod-balanced row split puts block p on rank p; no data-path collective).
+Workload: BASELINE.json configs[4] (config 5), the R-MAT(0.45, 0.15, 0.15, 0.25) graph at scale 22,
+edge factor 16 (4.19 M rows, 67 M nnz, 2.5e9 intermediate products, nnz(C) 2.5e9 > 2^31),
+fp32 — the largest configuration quoted at 1/2/4/8 GPUs that fits one B200 with room for the
+bench's own buffers (scale 23: 40.5 GB peak, 0.3 s per step).  One step = the whole
+hot path of SURVEY.md §8(a) on one input already resident in HBM: symbolic (n_prod, grouping,
+hash count, scan) -> exact allocation of C -> numeric (grouping, accumulate, gather, sort, write).
 
-Timing: W untimed warm-ups; K timed steps, each bracketed by CUDA events on the handle's
-stream, the L2 flushed (512 MiB write) before every step outside the events; barrier +
-synchronize on both sides; max over ranks.  `e2e` re-times the step through the public
-Python API from pinned HOST buffers: H2D of A, the step, and D2H of all of C.
+N GPUs (torchrun, one rank per GPU, NCCL): the rows of C are independent, so the
+SAME matrix is split into n_prod-balanced row blocks (strong scaling): rank 0
+holds A, B = A is broadcast in chunks (NCCL), every rank computes the same split points on its GPU,
+multiplies its zero-copy row block, and the nnz counts are all-gathered (dist.py).  `value` times
+the per-rank step (the local two-phase SpGEMM), max over ranks; `e2e` adds the host->device copy,
+the broadcast, the partition, the all-gather and the device->host copy of every rank's C block.
 
-`--impl reference`: the CPU oracle (oracle/, plain C Gustavson, 1 core) on the same
-config, rank 0 only — the reference arm of this tier (there is no reference library).
+Timing: W untimed warm-ups; K timed steps, CUDA events on the handle's stream, L2 flushed (512 MiB
+write) before every step outside the events (A is 0.54 GB, C 20 GB: larger than L2 anyway);
+barrier + synchronize on both sides; max over ranks; nvidia-smi clocks sampled during the steps.
+Attribution (roofline): one more step with the per-group kernels serialised on one stream and
+timed per group (CUDA events): the dominant kernel is the group with the largest time; its
+algorithmic bytes (SURVEY.md §8(d) streaming model) / its time = `roofline.achieved`.
+
+`--impl reference`: the CPU oracle (oracle/, plain C Gustavson, row-parallel over the host's
+cores) on a bounded sample of the same workload, rank 0 only.
 """
 from __future__ import annotations
 
@@ -41,6 +50,7 @@ REASON_BITS = {  # nvidia-smi clocks_event_reasons bitmask
     0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
     0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
 }
+PER_CONFIG = [("cant", "f32"), ("cant", "f64"), ("webbase", "f32")]
 
 
 def parse():
@@ -49,13 +59,11 @@ def parse():
     p.add_argument("--steps", type=int, default=10)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", default="cant")
+    p.add_argument("--config", default="rmat22")
     p.add_argument("--dtype", default="f32", choices=["f32", "f64"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--cpu-runs", type=int, default=5)
-    p.add_argument("--lanes", type=int, default=0, help="lanes per B row (0 = library auto)")
-    p.add_argument("--streams", type=int, default=1)
+    p.add_argument("--no-per-config", action="store_true")
     p.add_argument("--opt", action="append", default=[],
                    help="library option name=value (ablations, e.g. rank_acc=0; see _lib.OPTIONS)")
     return p.parse_args()
@@ -65,19 +73,21 @@ def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
 
-def workload(args, rank):
+def workload(config, dtype):
     import synth
-    A = synth.config(args.config, "uniform", seed=rank)
-    dt = np.float32 if args.dtype == "f32" else np.float64
+    A = synth.config(config, "uniform", 7)
+    dt = np.float32 if dtype == "f32" else np.float64
     return A.astype(dt), dt
 
 
 def config_dict(args, A, world):
-    return {"workload": f"{args.config}-like A^2" if args.config != "poisson64" else "poisson64 A^2",
-            "matrix": A.name, "rows": A.m, "nnz_a": A.nnz, "dtype": args.dtype,
-            "per_rank": "row block p of diag(A_0..A_{N-1})^2 (weak scaling)" if world > 1 else "single GPU",
-            "l2": "flushed (512 MiB write) before every timed step", "inputs": "device-resident (value)",
-            **({"options": dict(o.split("=") for o in args.opt)} if getattr(args, "opt", None) else {})}
+    return {"workload": f"{args.config} A^2", "matrix": A.name, "rows": A.m, "nnz_a": A.nnz,
+            "dtype": args.dtype, "baseline_config": "BASELINE.json configs[4] (config 5)" if args.config.startswith("rmat")
+            else "BASELINE.json configs[1..3]",
+            "partition": "n_prod-balanced row blocks of one matrix (strong scaling)" if world > 1 else "single GPU",
+            "l2": "flushed (512 MiB write) before every timed step; inputs larger than L2",
+            "inputs": "device-resident (value)",
+            **({"options": dict(o.split("=") for o in args.opt)} if args.opt else {})}
 
 
 # ----------------------------------------------------------------------------- clocks
@@ -131,7 +141,7 @@ class ClockSampler:
 
 # ----------------------------------------------------------------------------- roofline model
 def algorithmic_bytes(st: dict, phase: str, g: int, vbytes: int) -> int:
-    """SURVEY.md §8(d) / DESIGN.md §6 streaming model (no reuse), per group launch:
+    """SURVEY.md §8(d) streaming model (no reuse), per group launch:
     symbolic: 4 B/product (col_B) + 20 B/nnz(A) (col_A + rpt_B pair) + 28 B/row;
     numeric: (4+s) B/product (col_B,val_B) + (20+s) B/nnz(A) + (4+s) B/nnz(C) write + 36 B/row."""
     if phase == "sym":
@@ -140,84 +150,126 @@ def algorithmic_bytes(st: dict, phase: str, g: int, vbytes: int) -> int:
             + (4 + vbytes) * st["num_nnzc"][g] + 36 * st["num_rows"][g])
 
 
-def kernel_name(phase: str, g: int, kind: int = 0) -> str:
-    """Group -> kernel template as it appears in ncu / cuobjdump (spgemm_internal.cuh group ids;
-    kind = spgemm_kernel_t the library reports for the group)."""
-    if phase == "sym":
-        k = {2: "k_sym_rankcnt<TPR,UPPER,KP,MC>", 3: "k_sym_range", 5: "k_sym_global"}.get(kind, "k_sym_smem<T,TPR,BS,OPT>")
-        return f"{k} (group {g})"
-    k = {2: "k_num_rankacc<VT,TPR,UPPER,KP,MC>", 3: "k_num_range<VT>", 4: "k_num_cluster<VT,CS>",
-         5: "k_num_global<VT>", 6: "k_num_rankbig<VT>"}.get(kind, "k_num_smem<VT,T,TPR,BS,UPPER>")
-    return f"{k} (group {g})"
+FAMILY = {1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big", 7: "tiny", 8: "batch", 9: "esc"}
+SYM_KERNEL = {1: "k_sym_smem", 2: "k_sym_rankcnt", 3: "k_sym_range_bits", 5: "k_sym_global", 7: "k_sym_tiny",
+              8: "k_sym_batch"}
+NUM_KERNEL = {1: "k_num_smem", 2: "k_num_rankacc", 3: "k_num_range", 4: "k_num_cluster", 5: "k_num_global",
+              6: "k_num_rankbig", 7: "k_num_tiny", 9: "k_num_esc"}
 
 
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy bandwidth)"
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def load_traffic(phase, g, dtype):
-    p = os.path.join(ROOT, "profiles", "traffic.json")
+def load_traffic(config, dtype, phase, g):
+    """DRAM bytes of this group's launch from the committed ncu capture of the same config
+    (profiles/traffic_r02.json, written by scripts/traffic.py), or None."""
+    p = os.path.join(ROOT, "profiles", "traffic_r02.json")
     if not os.path.exists(p):
-        return None
+        return None, None
     d = json.load(open(p))
-    return d.get(f"{phase}_g{g}_{dtype}")
+    e = d.get(f"{config}|{dtype}|{phase}|g{g}")
+    return (e["dram_bytes"], e["source"]) if e else (None, None)
 
 
 # ----------------------------------------------------------------------------- reference arm
+def reference_sample(A, nprod_rows, frac):
+    """Rows [0, r) of A holding about `frac` of the intermediate products (hubs included)."""
+    import oracle
+    cum = np.cumsum(nprod_rows)
+    r = int(np.searchsorted(cum, frac * cum[-1])) + 1
+    return oracle.row_slice(A, 0, min(r, A.m)), int(cum[min(r, A.m) - 1])
+
+
 def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import oracle
-    A, dt = workload(args, 0)
-    _, total = oracle.nprod(A, A)
+    A, dt = workload(args.config, args.dtype)
+    nprod_rows, total = oracle.nprod(A, A)
+    S, s_nprod = reference_sample(A, nprod_rows, 1.0 / 8)
     oracle.build()
     times = []
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        oracle.spgemm(A, A, dt)
+        oracle.spgemm(S, A, dt, parallel=True, with_abs=False)
         t = time.perf_counter() - t0
         if i >= args.warmup:
             times.append(t)
     tot = sum(times)
-    val = 2 * total * len(times) / tot / 1e9
+    val = 2 * s_nprod * len(times) / tot / 1e9
+    sample = (f"rows [0, {S.m}) of {A.name} (1/8 of its {total} products: {s_nprod}) times A, "
+              f"row-parallel oracle on {oracle.threads()} threads, per step")
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": config_dict(args, A, 1), "impl": "reference",
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"full {A.name} A^2 per step (nprod {total})"},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": oracle.threads(), "kind": "oracle", "sample": sample},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ----------------------------------------------------------------------------- our arm
+def csr_bytes(M, vbytes):
+    return M.rpt.numel() * 8 + M.col.numel() * 4 + (M.val.numel() * vbytes if M.val is not None else 0)
+
+
+def quick_value(P, torch, dev, config, dtype, steps, flush, opts):
+    """GFLOPS of `config` on this GPU (graphs on, L2 flushed), for the per_config block."""
+    A, dt = workload(config, dtype)
+    tdt = torch.float32 if dt == np.float32 else torch.float64
+    dA = P.CsrMatrix.from_host(A, dev, tdt)
+    h = P.Handle(dev)
+    for k, v in opts:
+        h.set_option(k, v)
+    for _ in range(3):
+        h.multiply(dA, dA)
+    torch.cuda.synchronize()
+    ms = []
+    for _ in range(steps):
+        with torch.cuda.stream(h.stream):
+            flush.add_(1)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(h.stream)
+        C = h.multiply(dA, dA)
+        e1.record(h.stream)
+        e1.synchronize()
+        ms.append(e0.elapsed_time(e1))
+        del C
+    nprod = h.nprod
+    h.close()
+    t = statistics.median(ms)
+    return {"value": 2 * nprod / t / 1e6, "unit": UNIT, "ms_per_step": t, "steps": steps, "nprod": int(nprod)}
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
 
     rank, world, local = dist_env()
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+        backend = os.environ.get("BENCH_BACKEND", "nccl")  # gloo: multi-rank test on one GPU
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    torch.cuda.set_device(local if torch.cuda.device_count() > local else 0)
+    dev = torch.device("cuda", torch.cuda.current_device())
     import paper_conf_icpp_nagasakanm17_b200 as P
+    from paper_conf_icpp_nagasakanm17_b200 import dist as D
 
-    A, dt = workload(args, rank)
+    opts = [(k, int(v)) for k, v in (o.split("=") for o in args.opt)]
+    A, dt = workload(args.config, args.dtype)  # every rank builds the seeded host copy (for e2e)
     tdt = torch.float32 if dt == np.float32 else torch.float64
     vbytes = 4 if dt == np.float32 else 8
     h = P.Handle(dev)
-    # per-group kernel events over the timed region (timing=2 runs the group kernels eagerly; the
-    # CUDA-graph replay mode is timed separately below and reported as `graph_replay`)
-    h.set_option("lanes", args.lanes).set_option("streams", args.streams).set_option("timing", 2)
-    for o in args.opt:
-        k, v = o.split("=")
-        h.set_option(k, int(v))
-    dA = P.CsrMatrix.from_host(A, dev, tdt)
+    for k, v in opts:
+        h.set_option(k, v)
     stream = h.stream
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
@@ -226,105 +278,153 @@ def run_ours(args):
             dist.barrier()
         torch.cuda.synchronize()
 
+    def maxr(x):
+        t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sumr(x):
+        t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    # setup (untimed): A on rank 0's GPU, chunked broadcast of B = A, n_prod-balanced split
+    dA0 = P.CsrMatrix.from_host(A, dev, tdt) if rank == 0 else None
+    barrier()
+    t0 = time.perf_counter()
+    Bd = D.broadcast_csr(dA0, 0, dev, tdt) if world > 1 else dA0
+    barrier()
+    bcast_s = time.perf_counter() - t0
+    splits = D.cuda_partition(h)(Bd, Bd, world)
+    r0, r1 = splits[rank], splits[rank + 1]
+    mine = D.row_slice(Bd, r0, r1)
+
     def step():
-        return h.multiply(dA, dA)
+        return h.multiply(mine, Bd)
 
     for _ in range(max(3, args.warmup)):
         step()
     barrier()
-
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    per_step_stats = []
     launches = 0
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev.index) as clk:
         barrier()
         t_wall = time.perf_counter()
         for i in range(args.steps):
             with torch.cuda.stream(stream):
-                flush.fill_(i & 0xFF)
+                flush.add_(1)
             ev[i][0].record(stream)
             C = step()
             ev[i][1].record(stream)
-            st = h.stats()  # waits for this step's events (per-group kernel timings)
-            per_step_stats.append(st)
+            st = h.stats()
             launches += st["kernel_launches_symbolic"] + st["kernel_launches_numeric"]
             del C
         barrier()
         t_wall = time.perf_counter() - t_wall
     step_ms = [a.elapsed_time(b) for a, b in ev]
-    tot_ms = sum(step_ms)
-    st = per_step_stats[-1]
-    nprod = st["nprod"]
-    tot_t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(tot_t, op=dist.ReduceOp.MAX)
-        np_t = torch.tensor([nprod], dtype=torch.float64, device=dev)
-        dist.all_reduce(np_t, op=dist.ReduceOp.SUM)
-        total_nprod = float(np_t.item())
-    else:
-        total_nprod = float(nprod)
-    max_ms = float(tot_t.item())
+    my_ms = sum(step_ms)
+    my_nprod = h.nprod
+    max_ms = maxr(my_ms)
+    total_nprod = sumr(my_nprod)
     value = 2 * total_nprod * args.steps / (max_ms / 1e3) / 1e9
+    imbalance = {"nprod_max_over_mean": maxr(my_nprod) / (total_nprod / world),
+                 "time_max_over_mean": max_ms / (sumr(my_ms) / world)}
 
-    # dominant kernel: group launch with the largest mean time across the timed steps
-    cand = {}
-    for s in per_step_stats:
-        for ph, key in (("sym", "sym_group_ms"), ("num", "num_group_ms")):
-            for g, ms in enumerate(s[key]):
-                if ms > 0:
-                    cand.setdefault((ph, g), []).append(ms)
-    (ph, g), mss = max(cand.items(), key=lambda kv: statistics.mean(kv[1]))
-    k_ms = statistics.mean(mss)
-    bytes_alg = algorithmic_bytes(st, ph, g, vbytes)
+    # attribution: one step with the group kernels serialised and timed per group
+    h.set_option("streams", 0).set_option("timing", 2)
+    with torch.cuda.stream(stream):
+        flush.add_(1)
+    C = step()
+    torch.cuda.synchronize()
+    sa = h.stats()
+    del C
+    h.set_option("streams", 1).set_option("timing", 1)
+    serial_ms = sa["setup_ms"] + sa["symbolic_ms"] + sa["scan_ms"] + sa["numeric_ms"]
+    groups = []
+    for ph, key, kk in (("sym", "sym_group_ms", "sym_kernel"), ("num", "num_group_ms", "num_kernel")):
+        for g, ms in enumerate(sa[key]):
+            if ms > 0:
+                groups.append((ms, ph, g, sa[kk][g]))
+    groups.sort(reverse=True)
+    k_ms, ph, g, kind = groups[0]
+    bytes_alg = algorithmic_bytes(sa, ph, g, vbytes)
     peak, peak_src = load_peaks()
     achieved = bytes_alg / (k_ms / 1e3) / 1e9
+    traffic, traffic_src = load_traffic(args.config, args.dtype, ph, g)
+    kname = (SYM_KERNEL if ph == "sym" else NUM_KERNEL).get(kind, "?")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": load_traffic(ph, g, args.dtype),
-                "kernel": kernel_name(ph, g, st["sym_kernel" if ph == "sym" else "num_kernel"][g]), "phase": ph, "group": g,
-                "launch_ms": k_ms, "share_of_step": k_ms / (tot_ms / args.steps),
-                "algorithmic_bytes_per_launch": bytes_alg, "peak_source": peak_src}
+                "traffic": traffic, "traffic_source": traffic_src,
+                "achieved_model": "algorithmic bytes (SURVEY.md §8(d) streaming model, no reuse: B-row re-reads "
+                                  "that hit L2 count as HBM bytes) / kernel time",
+                "frac_dram": (traffic / (k_ms / 1e3) / 1e9 / peak) if traffic else None,
+                "kernel": f"{kname} ({FAMILY.get(kind, '?')}, {ph} group {g})", "phase": ph, "group": g,
+                "launch_ms": k_ms, "share_of_serial_step": k_ms / serial_ms,
+                "algorithmic_bytes_per_launch": int(bytes_alg), "peak_source": peak_src,
+                "attribution": "per-group CUDA events, group kernels serialised on one stream (one extra step)",
+                "top_groups": [{"phase": p, "group": q, "kernel": (SYM_KERNEL if p == "sym" else NUM_KERNEL).get(k, "?"),
+                                "ms": m} for m, p, q, k in groups[:6]]}
 
-    # the same step with the captured phase segments replayed as CUDA graphs (timing=1)
-    h.set_option("timing", 1)
-    for _ in range(max(3, args.warmup)):
-        step()
-    barrier()
-    gev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    replays = 0
-    for i in range(args.steps):
-        with torch.cuda.stream(stream):
-            flush.fill_(i & 0xFF)
-        gev[i][0].record(stream)
-        C = step()
-        gev[i][1].record(stream)
-        replays += h.stats()["graph_replays"]
+    # measured peak device memory of one step (all library workspace through torch's allocator)
+    peak_mem = None
+    if world == 1:
+        hp = P.Handle(dev, torch_allocator=True)
+        for k, v in opts:
+            hp.set_option(k, v)
+        del flush
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+        free0 = torch.cuda.mem_get_info(dev)[0]
+        torch.cuda.reset_peak_memory_stats(dev)
+        base = torch.cuda.memory_allocated(dev)
+        C = hp.multiply(mine, Bd)
+        torch.cuda.synchronize()
+        peak_alloc = torch.cuda.max_memory_allocated(dev)
+        a_bytes = csr_bytes(Bd, vbytes)
+        c_bytes = csr_bytes(C, vbytes)
+        peak_mem = {"peak_device_bytes": int(peak_alloc), "inputs_bytes": int(a_bytes), "c_bytes": int(c_bytes),
+                    "overhead_bytes": int(peak_alloc - a_bytes - c_bytes),
+                    "step_increase_bytes": int(peak_alloc - base),
+                    "cudaMemGetInfo_free_drop_bytes": int(free0 - torch.cuda.mem_get_info(dev)[0]),
+                    "how": "torch.cuda.max_memory_allocated over one step, library workspace through the torch "
+                           "allocator callbacks (include/spgemm.h spgemm_allocator_t); inputs resident, "
+                           "no other buffers"}
         del C
-    barrier()
-    g_ms = sum(a.elapsed_time(b) for a, b in gev)
-    gt = torch.tensor([g_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(gt, op=dist.ReduceOp.MAX)
-    graph_replay = {"value": 2 * total_nprod * args.steps / (float(gt.item()) / 1e3) / 1e9, "unit": UNIT,
-                    "ms_per_step": float(gt.item()) / args.steps, "segments_replayed": int(replays)}
+        hp.close()
+        flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
-    # end to end through the public API from pinned host buffers
+    # end to end through the public API: pinned host A -> device, (broadcast, split,) multiply,
+    # device -> pinned host C block
     e2e = None
     if not args.no_e2e:
-        hA = P.CsrMatrix.from_host(A, None, tdt, pin=True)
-        bi = hA.rpt.numel() * 8 + hA.col.numel() * 4 + hA.val.numel() * vbytes
-        e_ms, bo = [], 0
+        hA = P.CsrMatrix.from_host(A, None, tdt, pin=True) if rank == 0 else None
+        bi = csr_bytes(hA, vbytes) if rank == 0 else 0
+        nnz_mine = h.nnz_c
+        out = (torch.empty(r1 - r0 + 1, dtype=torch.int64, pin_memory=True),
+               torch.empty(nnz_mine, dtype=torch.int32, pin_memory=True),
+               torch.empty(nnz_mine, dtype=tdt, pin_memory=True))
+        bo = sum(x.numel() * x.element_size() for x in out)
+        e_ms = []
         for i in range(args.warmup + args.steps):
             with torch.cuda.stream(stream):
-                flush.fill_(i & 0xFF)
+                flush.add_(1)
+            barrier()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             with torch.cuda.stream(stream):
-                dA2 = hA.to(dev, non_blocking=True)
-            C = h.multiply(dA2, dA2)
+                dA2 = hA.to(dev, non_blocking=True) if rank == 0 else None
+            if world > 1:
+                with torch.cuda.stream(stream):
+                    B2 = D.broadcast_csr(dA2, 0, dev, tdt)
+                    sp = D.cuda_partition(h)(B2, B2, world)
+            else:
+                B2, sp = dA2, [0, A.m]
+            C = h.multiply(D.row_slice(B2, sp[rank], sp[rank + 1]), B2)
             with torch.cuda.stream(stream):
-                out = (torch.empty(C.rpt.shape, dtype=C.rpt.dtype, pin_memory=True),
-                       torch.empty(C.col.shape, dtype=C.col.dtype, pin_memory=True),
-                       torch.empty(C.val.shape, dtype=C.val.dtype, pin_memory=True))
+                if world > 1:
+                    cnt = torch.tensor([C.nnz], dtype=torch.int64, device=dev)
+                    dist.all_gather([torch.zeros_like(cnt) for _ in range(world)], cnt)
                 out[0].copy_(C.rpt, non_blocking=True)
                 out[1].copy_(C.col, non_blocking=True)
                 out[2].copy_(C.val, non_blocking=True)
@@ -332,42 +432,56 @@ def run_ours(args):
             e1.synchronize()
             if i >= args.warmup:
                 e_ms.append(e0.elapsed_time(e1))
-                bo = sum(x.numel() * x.element_size() for x in out)
-            del C, dA2, out
-        et = torch.tensor([sum(e_ms)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(et, op=dist.ReduceOp.MAX)
-        e2e = {"value": 2 * total_nprod * len(e_ms) / (float(et.item()) / 1e3) / 1e9, "unit": UNIT,
-               "h2d_bytes_per_step": int(bi), "d2h_bytes_per_step": int(bo),
-               "ms_per_step": float(et.item()) / len(e_ms)}
+            del C, dA2, B2
+        et = maxr(sum(e_ms))
+        e2e = {"value": 2 * total_nprod * len(e_ms) / (et / 1e3) / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": int(bi), "d2h_bytes_per_step": int(bo), "ms_per_step": et / len(e_ms),
+               "includes": "H2D of A (rank 0), " + ("NCCL broadcast, partition, all-gather of nnz, " if world > 1 else "")
+                           + "the step, D2H of the rank's C block (max over ranks)"}
+        del out
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
         oracle.build()
-        ts = []
-        for _ in range(args.cpu_runs):
-            t0 = time.perf_counter()
-            oracle.spgemm(A, A, dt)
-            ts.append(time.perf_counter() - t0)
-        cpu = {"value": 2 * nprod * len(ts) / sum(ts) / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"full {A.name} A^2 ({args.dtype}) x {len(ts)} runs, {sum(ts):.1f} s"}
+        t0 = time.perf_counter()
+        oracle.spgemm(A, A, dt, parallel=True, with_abs=False)
+        t_all = time.perf_counter() - t0
+        nprod_rows, _ = oracle.nprod(A, A)
+        S, s_nprod = reference_sample(A, nprod_rows, 1.0 / 64)
+        t0 = time.perf_counter()
+        oracle.spgemm(S, A, dt)
+        t_one = time.perf_counter() - t0
+        cpu = {"value": 2 * my_nprod / t_all / 1e9, "unit": UNIT, "cores": oracle.threads(), "kind": "oracle",
+               "sample": f"full {A.name} A^2 ({args.dtype}), 1 run of the row-parallel oracle "
+                         f"({oracle.threads()} threads of {oracle.cores()} host cores), {t_all:.1f} s",
+               "single_thread": {"value": 2 * s_nprod / t_one / 1e9, "unit": UNIT, "cores": 1,
+                                 "sample": f"rows [0, {S.m}) (1/64 of the products) x A, {t_one:.1f} s"}}
 
-    a_bytes = (A.m + 1) * 8 + A.nnz * (4 + vbytes)  # B = A shares these buffers
-    c_bytes = (A.m + 1) * 8 + int(st["nnz_c"]) * (4 + vbytes)
-    phases = {k: statistics.median([s[k] for s in per_step_stats]) for k in ("setup_ms", "symbolic_ms", "scan_ms", "numeric_ms")}
+    per_config = None
+    if rank == 0 and world == 1 and not args.no_per_config:
+        per_config = {}
+        for cfg, dty in PER_CONFIG:
+            if (cfg, dty) != (args.config, args.dtype):
+                per_config[f"{cfg}_{dty}"] = quick_value(P, torch, dev, cfg, dty, 10, flush, opts)
+
+    phases = {k: sa[k] for k in ("setup_ms", "symbolic_ms", "scan_ms", "numeric_ms")}
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": max_ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+                "scaling": "strong", "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
                 "config": config_dict(args, A, world), "impl": "ours",
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "graph_replay": graph_replay,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk.summary(),
-                "nprod": int(total_nprod), "nnz_c": int(st["nnz_c"]), "phase_ms_median": phases,
-                "step_ms": step_ms, "wall_s": t_wall,
-                "peak_mem_bytes": int(a_bytes + c_bytes + max(s["workspace_peak_bytes"] for s in per_step_stats)),
-                "workspace_peak_bytes": int(max(s["workspace_peak_bytes"] for s in per_step_stats))}
+                "nprod": int(total_nprod), "nnz_c": int(sumr(h.nnz_c)),
+                "phase_ms_serial_step": phases, "step_ms": step_ms, "wall_s": t_wall,
+                "peak_mem": peak_mem, "workspace_peak_bytes": int(st["workspace_peak_bytes"]),
+                "multi_gpu": {"ranks": world, "splits": [int(x) for x in splits], "broadcast_s": bcast_s,
+                              "imbalance": imbalance} if world > 1 else None,
+                "per_config": per_config}
         print(json.dumps(line), flush=True)
+    else:
+        sumr(h.nnz_c)
     h.close()
     if world > 1:
         dist.destroy_process_group()

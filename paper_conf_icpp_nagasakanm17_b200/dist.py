@@ -4,7 +4,7 @@ Rows of C are independent (Alg. 1 loops over rows of A), so the onl
 steps are replicating B (and A when it lives on one rank) and exchanging the per-rank nnz(C)
 counts.  One process per GPU (torch.distributed, NCCL over NVLink/NVSwitch):
 
-  1. broadcast B (and A) from `src` — the sizes first, then rpt / col / val;
+  1. broadcast B (and A) from `src` — the sizes first, then rpt / col / val in 64 MB chunks;
   2. every rank computes the same n_prod-balanced split points (spgemm_row_partition, on its
      own GPU — no collective needed, the splits agree by construction);
   3. rank p runs the two-phase SpGEMM on rows [s_p, s_{p+1}) of A as a zero-copy slice
@@ -39,7 +39,22 @@ class ShardResult:
     splits: list
 
 
-def _bcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None) -> CsrMatrix:
+BCAST_CHUNK_BYTES = 64 << 20  # NCCL broadcast granularity (many in flight; large tensors pipelined)
+
+
+def _bcast_chunked(t: torch.Tensor, src: int, group=None, chunk_bytes: int = BCAST_CHUNK_BYTES) -> None:
+    """Broadcast a contiguous tensor in chunks (asynchronous ops, waited together), so a
+    gigabyte-sized B is pipelined through the collective instead of one monolithic call."""
+    flat = t.view(-1)
+    per = max(1, chunk_bytes // max(1, t.element_size()))
+    works = [dist.broadcast(flat[i:i + per], src, group=group, async_op=True) for i in range(0, flat.numel(), per)]
+    for w in works:
+        w.wait()
+
+
+def broadcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None) -> CsrMatrix:
+    """Replicate a CSR matrix held by rank `src` on every rank of `group` (sizes first, then
+    rpt / col / val in chunks)."""
     rank = dist.get_rank(group)
     meta = torch.zeros(3, dtype=torch.int64, device=device)
     if rank == src:
@@ -54,8 +69,11 @@ def _bcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None) -> C
         val = torch.empty(nnz, dtype=dtype, device=device)
     for t in (rpt, col, val):
         if t.numel():
-            dist.broadcast(t, src, group=group)
+            _bcast_chunked(t, src, group)
     return CsrMatrix(m, n, rpt, col, val)
+
+
+_bcast_csr = broadcast_csr
 
 
 def row_slice(A: CsrMatrix, r0: int, r1: int) -> CsrMatrix:

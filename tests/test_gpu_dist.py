@@ -62,3 +62,29 @@ def test_two_rank_row_partition(tmp_path, name):
     assert np.array_equal(np.concatenate([s["col"] for s in sh]), r_col)
     assert np.array_equal(np.concatenate([s["val"] for s in sh]), r_val)
     assert sum(int(s["nprod"]) for s in sh) == total
+
+
+def test_bench_sharded_two_ranks_gloo(tmp_path):
+    """bench.py's N>1 path (broadcast of B, n_prod-balanced split, per-rank multiply, all-gather,
+    max over ranks, e2e) with two ranks on one GPU over gloo (the driver runs it over NCCL on one GPU
+    per rank); the two ranks' products must add up to the whole matrix's n_prod."""
+    import json
+    import subprocess
+    import sys
+    import oracle
+    import synth
+    if not torch.cuda.is_available():
+        pytest.fail("needs a GPU")
+    env = dict(os.environ, BENCH_BACKEND="gloo")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                        "--master-addr", "127.0.0.1", "--master-port", str(_port()), os.path.join(ROOT, "bench.py"),
+                        "--gpus", "2", "--steps", "2", "--warmup", "1", "--config", "rmat16"],
+                       capture_output=True, text=True, env=env, cwd=ROOT, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    line = json.loads([x for x in r.stdout.splitlines() if x.startswith("{")][-1])
+    A = synth.config("rmat16", "uniform", 7)
+    _, total = oracle.nprod(A, A)
+    assert line["n_gpus"] == 2 and line["nprod"] == total and line["scaling"] == "strong"
+    sp = line["multi_gpu"]["splits"]
+    assert sp[0] == 0 and sp[-1] == A.m and len(sp) == 3
+    assert line["e2e"]["value"] > 0 and line["gpu_launches"] > 0
