@@ -469,26 +469,20 @@ def test_row_partition(spg):
             assert s.tolist() == want
 
 
-# ------------------------------------------------------------------ full size, sampled
+# ------------------------------------------------------------------ config 5 at full size
 
 @pytest.mark.slow
-def test_rmat_s20_sampled(spg):
+def test_rmat_s20_full(spg):
+    """R-MAT s20 (config 5's shape at 1/4 size): full rpt and every row against the oracle."""
     A = synth.rmat(20).with_values("uniform", 7)
-    with spg.Handle() as h:
-        dA = _dev(spg, A, np.float32)
-        C = h.multiply(dA, dA)
-        rpt, col, val = C.numpy()
     A32 = A.astype(np.float32)
-    assert rpt[0] == 0 and np.all(np.diff(rpt) >= 0)
-    rng = np.random.default_rng(0)
-    heavy = np.argsort(np.diff(rpt))[-20:]
-    for r in np.concatenate([rng.integers(0, A.m, 200), heavy]):
-        S = oracle.row_slice(A32, int(r), int(r) + 1)
-        r_rpt, r_col, r_val, r_abs = oracle.spgemm(S, A32, np.float32)
-        s, e = rpt[r], rpt[r + 1]
-        assert e - s == r_rpt[1]
-        assert np.array_equal(col[s:e], r_col)
-        assert np.all(np.abs(val[s:e] - r_val) <= 1e-5 * r_abs)
+    with spg.Handle() as h:
+        dA = _dev(spg, A32, np.float32)
+        C = h.multiply(dA, dA)
+        torch.cuda.synchronize()
+        rpt = C.rpt.cpu().numpy()
+        assert np.array_equal(rpt, oracle.symbolic_omp(A32, A32))
+        _chunked_full_parity(C, A32, rpt, 1e-5)
 
 
 def _sampled_rows_parity(C, A32, rows, rtol):
@@ -507,10 +501,32 @@ def _sampled_rows_parity(C, A32, rows, rtol):
     return rpt
 
 
+def _chunked_full_parity(C, A32, rpt, rtol, max_entries=200_000_000):
+    """Every row of a device C against the row-parallel oracle, in row blocks of at most
+    `max_entries` output entries (C may be tens of GB): col bit-exact, values within rtol * S."""
+    r0 = 0
+    while r0 < A32.m:
+        r1 = int(np.searchsorted(rpt, rpt[r0] + max_entries, side="right")) - 1
+        r1 = min(A32.m, max(r1, r0 + 1))
+        S = oracle.row_slice(A32, r0, r1)
+        c_rpt, c_col, c_val, c_abs = oracle.spgemm(S, A32, np.float32, parallel=True)
+        s, e = int(rpt[r0]), int(rpt[r1])
+        assert np.array_equal(c_rpt + s, rpt[r0:r1 + 1]), f"rows [{r0}, {r1}): rpt"
+        col = C.col[s:e].cpu().numpy()
+        assert np.array_equal(col, c_col), f"rows [{r0}, {r1}): col differs"
+        val = C.val[s:e].cpu().numpy().astype(np.float64)
+        bad = np.abs(val - c_val.astype(np.float64)) > rtol * c_abs
+        assert not bad.any(), f"rows [{r0}, {r1}): {int(bad.sum())} values out of tolerance"
+        del col, val, c_col, c_val, c_abs
+        r0 = r1
+
+
 @pytest.mark.slow
-def test_rmat_s22_sampled(spg):
-    """Config 5 at full single-GPU size: R-MAT(0.45,0.15,0.15,0.25) s22 ef16, nnz(C) > 2^31
-    (int64 rpt path), sampled rows + heaviest rows against the oracle, global invariants."""
+def test_rmat_s22_full_parity(spg):
+    """Config 5 at full single-GPU size, EVERY row: R-MAT(0.45,0.15,0.15,0.25) s22 ef16, nnz(C) >
+    2^31 (int64 rpt path).  Full rpt against the row-parallel oracle's symbolic pass (Alg. 2 n_prod
+    total too), then every row's columns bit-exact and values within 1e-5 * S in row blocks; the
+    heaviest C rows (by C-row length) are in the blocks like every other row."""
     A = synth.rmat(22).with_values("uniform", 7)
     A32 = A.astype(np.float32)
     with spg.Handle() as h:
@@ -521,18 +537,32 @@ def test_rmat_s22_sampled(spg):
         _, total = oracle.nprod(A32, A32)
         assert h.nprod == total
         assert C.nnz > 2**31 - 1  # exercises 64-bit row pointers / output offsets
-        rng = np.random.default_rng(1)
-        lens = (A.rpt[1:] - A.rpt[:-1])
-        heavy = np.argsort(lens)[-8:]
-        rows = np.concatenate([rng.integers(0, A.m, 60), heavy, [0, A.m - 1]])
-        rpt = _sampled_rows_parity(C, A32, rows, 1e-5)
-        assert rpt[0] == 0 and np.all(np.diff(rpt) >= 0) and rpt[-1] == C.nnz
-        # every output row strictly increasing: device-side check over all of C
-        d = C.col[1:].to(torch.int64) - C.col[:-1].to(torch.int64)
-        starts = torch.zeros(C.nnz, dtype=torch.bool, device=C.col.device)
-        starts[C.rpt[1:-1][C.rpt[1:-1] < C.nnz]] = True
-        assert bool(((d > 0) | starts[1:]).all())
-        assert st["nnz_c"] == C.nnz
+        rpt = C.rpt.cpu().numpy()
+        assert np.array_equal(rpt, oracle.symbolic_omp(A32, A32)), "rpt differs from the oracle"
+        assert st["nnz_c"] == C.nnz == rpt[-1]
+        assert any(st["num_kernel"][g] == 9 for g in range(15, 22) if st["num_rows"][g]), "ESC rows expected at s22"
+        heavy = np.argsort(np.diff(rpt))[-8:]  # C-row length
+        assert np.diff(rpt)[heavy].min() > 8192  # rows beyond the CTA groups are part of the check
+        _chunked_full_parity(C, A32, rpt, 1e-5)
+
+
+@pytest.mark.slow
+def test_rmat_s23_rpt_and_heavy_rows(spg):
+    """Config 5 at its largest size (s23: nnz(C) 5.3e9, C 42 GB): full rpt against the oracle,
+    the 16 heaviest C rows and 48 random rows value-checked."""
+    A = synth.rmat(23).with_values("uniform", 7)
+    A32 = A.astype(np.float32)
+    with spg.Handle() as h:
+        dA = _dev(spg, A32, np.float32)
+        C = h.multiply(dA, dA)
+        torch.cuda.synchronize()
+        rpt = C.rpt.cpu().numpy()
+        assert np.array_equal(rpt, oracle.symbolic_omp(A32, A32)), "rpt differs from the oracle"
+        _, total = oracle.nprod(A32, A32)
+        assert h.nprod == total
+        rng = np.random.default_rng(3)
+        rows = np.concatenate([np.argsort(np.diff(rpt))[-16:], rng.integers(0, A.m, 48)])
+        _sampled_rows_parity(C, A32, rows, 1e-5)
 
 
 # ------------------------------------------------------------------ rank-indexed accumulation
