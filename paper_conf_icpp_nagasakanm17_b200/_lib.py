@@ -10,7 +10,8 @@ import os
 from ctypes import POINTER, c_char_p, c_float, c_int, c_int32, c_int64, c_size_t, c_void_p
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libspgemm.so")
+# SPGEMM_LIB: an alternative build of the same library (diagnostics: kernel variants side by side)
+LIB_PATH = os.environ.get("SPGEMM_LIB") or os.path.join(_HERE, "libspgemm.so")
 
 SPGEMM_F32, SPGEMM_F64 = 0, 1
 MAX_GROUPS = 24

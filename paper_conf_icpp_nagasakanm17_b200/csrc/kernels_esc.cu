@@ -274,19 +274,23 @@ __device__ __forceinline__ int sw4(int j) { return j + (j >> 5); }
 template <typename VT>
 __device__ __forceinline__ int swv(int j) { return sizeof(VT) == 8 ? j + (j >> 4) : j + (j >> 5); }
 
-constexpr int kEscSkew = 16;  // a batch whose largest bucket holds more products is refined
+#ifndef SPG_ESC_SKEW
+#define SPG_ESC_SKEW 16
+#endif
+constexpr int kEscSkew = SPG_ESC_SKEW;  // a batch whose largest bucket holds more products is refined
 // BM: coarse buckets per row = BM * next_pow2(n_prod_i) (2, or 1 where shared memory is short);
 // REFINE: the skew refinement (its fine counters) fits
 
 template <typename VT, int TPR, int KP, int MC, int R, int BM, bool REFINE>
 struct NumEscSmem {
   static constexpr int CAP = TPR * KP;
-  int sk[CAP + CAP / 32 + 1];   // keys: bucket order, then sorted, then compacted output
-  VT sv[CAP + CAP / 16 + 1];    // values, same orders
   static constexpr int NB = BM * CAP;  // coarse (and fine) buckets per batch, at most
-  int cnt[NB + NB / 32 + 2];    // coarse bucket counters -> starts (-> fine base | bits << 24)
-  unsigned rs[CAP / 32 + 1];    // slot j starts a row
-  uint16_t sb[CAP];             // bucket of each slot (bucket order)
+  int sk[CAP + CAP / 32 + 1];   // keys: bucket order, then the compacted output
+  VT sv[CAP + CAP / 16 + 1];    // values, same orders
+  alignas(16) int cnt[NB + NB / 32 + 2];  // coarse bucket counters -> starts (-> fine base | bits << 24)
+  int db[NB + NB / 32 + 2];     // distinct entries per bucket -> output base | (bucket has equal keys) << 30
+  unsigned dupw[NB / 2 + 1];    // 16-bit counters: products with an equal key placed before them
+  uint16_t sb[CAP];             // bucket of each slot (bucket order); bit 15: the slot heads its key
   union {                       // the gather's metadata is dead once the products are in registers
     EscMeta<VT, TPR * MC, CAP> mt;
     int fcnt[REFINE ? NB + NB / 32 + 2 : 1];  // fine bucket counters -> starts (skewed batches)
@@ -328,15 +332,15 @@ __global__ __launch_bounds__(TPR, (1024 / TPR)) void k_num_esc(NumArgs a) {
   S* sm = reinterpret_cast<S*>(smem_raw);
   const int t = threadIdx.x;
   esc_rows<R, true>(&sm->rt, a.rows, a.nrows, a.a_rpt, a.nprod, a.rlohi, a.c_rpt);
-  for (int i = t; i < S::NB + S::NB / 32 + 2; i += TPR) sm->cnt[i] = 0;
-  for (int i = t; i < CAP / 32 + 1; i += TPR) sm->rs[i] = 0u;
+  {
+    int4* c4 = reinterpret_cast<int4*>(sm->cnt);
+    for (int i = t; i < (S::NB + S::NB / 32 + 2) / 4; i += TPR) c4[i] = make_int4(0, 0, 0, 0);
+    for (int i = ((S::NB + S::NB / 32 + 2) / 4) * 4 + t; i < S::NB + S::NB / 32 + 2; i += TPR) sm->cnt[i] = 0;
+    for (int i = t; i < S::NB / 2 + 1; i += TPR) sm->dupw[i] = 0u;
+  }
   if (t == 0) sm->smax = 0;
   __syncthreads();
   const int nr = sm->rt.nr;
-  if (t < nr) {
-    const int p0 = sm->rt.pbase[t];
-    atomicOr(&sm->rs[p0 >> 5], 1u << (p0 & 31));
-  }
   int key[KP], rix[KP];
   VT val[KP];
   esc_gather<VT, true, TPR, KP, MC, R, CAP>(&sm->rt, &sm->u.mt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
@@ -438,74 +442,90 @@ __global__ __launch_bounds__(TPR, (1024 / TPR)) void k_num_esc(NumArgs a) {
       sm->sb[slot] = (uint16_t)b;
     }
   __syncthreads();
-  // rank inside the bucket (PAPER.md:173's count of smaller keys; equal keys by slot), one slot
-  // per lane in bucket order: the lanes of a warp walk the same few buckets together (uniform
-  // trip counts, broadcast reads)
-  int np[KP];
+  // Inside the bucket, one slot per lane in bucket order (the lanes of a warp walk the same few
+  // buckets together: uniform trip counts, broadcast reads): lt = #smaller keys (PAPER.md:173's
+  // comparison rank), the slot heads its key when no equal key sits before it; a head sums the
+  // values of all equal keys (accumulation in the working precision); a non-head
+  // is counted as a duplicate of its bucket.
+  int lt[KP];
 #pragma unroll
   for (int i = 0; i < KP; ++i) {
     const int j = i * TPR + t;
-    np[i] = -1;
+    lt[i] = -1;
     if (j < Pt) {
       const int b = sm->sb[j];
       const int j0 = bst[sw4(b)], j1 = bst[sw4(b + 1)];
       const int k = sm->sk[sw4(j)];
-      int rk = 0;
+      VT sum = VT(0);
+      int l = 0, eqb = 0;
 #pragma unroll 1
       for (int q = j0; q < j1; ++q) {
         const int k2 = sm->sk[sw4(q)];
-        rk += (k2 < k) | ((k2 == k) & (q < j));
+        l += k2 < k;
+        if (k2 == k) {  // (rare for weakly compressing rows, except q == j)
+          eqb += q < j;
+          sum += sm->sv[swv<VT>(q)];
+        }
       }
-      np[i] = j0 + rk;
-      key[i] = k;
-      val[i] = sm->sv[swv<VT>(j)];
+      if (eqb == 0) {
+        lt[i] = l;
+        key[i] = k;
+        val[i] = sum;
+        sm->sb[j] = (uint16_t)(b | 0x8000);
+      } else {
+        atomicAdd(&sm->dupw[b >> 1], 1u << (16 * (b & 1)));
+      }
     }
   }
   __syncthreads();
-#pragma unroll
-  for (int i = 0; i < KP; ++i)
-    if (np[i] >= 0) {
-      sm->sk[sw4(np[i])] = key[i];
-      sm->sv[swv<VT>(np[i])] = val[i];
-    }
-  __syncthreads();
-  // heads: first slot of a row or a key change; blocked slots t*KP .. t*KP+KP-1
-  auto row_start = [&](int j) { return (sm->rs[j >> 5] >> (j & 31)) & 1u; };
-  unsigned hm = 0;
-  int nh = 0;
-#pragma unroll
-  for (int i = 0; i < KP; ++i) {
-    const int j = t * KP + i;
-    if (j < Pt && (row_start(j) || sm->sk[sw4(j - 1)] != sm->sk[sw4(j)])) {
-      hm |= 1u << i;
-      ++nh;
-    }
-  }
+  // distinct entries per bucket -> exclusive scan (blocked, KB buckets per thread) -> output base
   int H;
-  const int hbase = esc_scan<TPR>(nh, &H, sm->ws);
+  {
+    int d[KB], s = 0;
+#pragma unroll
+    for (int i = 0; i < KB; ++i) {
+      const int b = t * KB + i;
+      const int dup = (int)((sm->dupw[b >> 1] >> (16 * (b & 1))) & 0xffffu);
+      d[i] = (b < NBt ? bst[sw4(b + 1)] - bst[sw4(b)] : 0) - dup;
+      s += d[i];
+      d[i] |= dup ? (1 << 30) : 0;
+    }
+    int run = esc_scan<TPR>(s, &H, sm->ws);
+#pragma unroll
+    for (int i = 0; i < KB; ++i) {
+      sm->db[sw4(t * KB + i)] = run | (d[i] & (1 << 30));
+      run += d[i] & ~(1 << 30);
+    }
+  }
   const int Ot = sm->rt.obase[nr];
   const bool ok = H == Ot;  // CTA-uniform; false only when symbolic and numeric disagree
   if (!ok && t == 0) atomicOr(a.err_flags, 2);
+  __syncthreads();
+  // each head's position among the batch's distinct entries: its bucket's base + the number of
+  // distinct smaller keys in the bucket (= lt when the bucket holds no equal keys)
 #pragma unroll
   for (int i = 0; i < KP; ++i) {
-    if (hm & (1u << i)) {
-      const int j = t * KP + i;
-      const int k = sm->sk[sw4(j)];
-      VT v = sm->sv[swv<VT>(j)];
-      for (int j2 = j + 1; j2 < Pt && !row_start(j2) && sm->sk[sw4(j2)] == k; ++j2) v += sm->sv[swv<VT>(j2)];
-      key[i] = k;  // registers reused for the run's entry
-      val[i] = v;
+    if (lt[i] >= 0) {
+      const int j = i * TPR + t;
+      const int b = sm->sb[j] & 0x7fff;
+      const int dbb = sm->db[sw4(b)];
+      int dl = lt[i];
+      if (dbb & (1 << 30)) {  // bucket with equal keys: count the smaller heads only
+        const int j0 = bst[sw4(b)], j1 = bst[sw4(b + 1)];
+        dl = 0;
+#pragma unroll 1
+        for (int q = j0; q < j1; ++q) dl += (sm->sk[sw4(q)] < key[i]) & (sm->sb[q] >> 15);
+      }
+      lt[i] = (dbb & ~(1 << 30)) + dl;
     }
   }
   __syncthreads();
   if (ok) {
-    int o = hbase;
 #pragma unroll
     for (int i = 0; i < KP; ++i)
-      if (hm & (1u << i)) {
-        sm->sk[sw4(o)] = key[i];
-        sm->sv[swv<VT>(o)] = val[i];
-        ++o;
+      if (lt[i] >= 0) {
+        sm->sk[sw4(lt[i])] = key[i];
+        sm->sv[swv<VT>(lt[i])] = val[i];
       }
   }
   __syncthreads();
@@ -540,8 +560,12 @@ struct EscCfg {
 // symbolic groups 2..9: bounds 128, 256, 512, 1024, 2048, 4096, 8192, 16384
 constexpr EscCfg kEscSym[] = {{0, 0, 0}, {0, 0, 0}, {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
                               {256, 8, 2}, {256, 8, 2}, {512, 8, 2}, {1024, 8, 2}, {1024, 16, 1}};
-constexpr EscCfg kEscNum32[] = {{0, 0, 0},  {0, 0, 0},  {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
-                                {256, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
+#ifndef SPG_ESC_SMALL_TPR
+#define SPG_ESC_SMALL_TPR 256
+#endif
+constexpr int kEscSmallTpr = SPG_ESC_SMALL_TPR;
+constexpr EscCfg kEscNum32[] = {{0, 0, 0},  {0, 0, 0},  {kEscSmallTpr, 8, 2},  {kEscSmallTpr, 8, 2},  {kEscSmallTpr, 8, 2},
+                                {kEscSmallTpr, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
 constexpr EscCfg kEscNum64[] = {{0, 0, 0},  {0, 0, 0},  {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
                                 {256, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
 template <typename VT>
@@ -619,7 +643,7 @@ bool numeric_esc_supported(int sym_group, bool fp64) {
   switch (sym_group) {
 #define SPG_G(I) \
   case I: return (fp64 ? num_esc_smem_g<double, I>() : num_esc_smem_g<float, I>()) <= kSmemLimit - 1024;
-    SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+    SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7)
 #undef SPG_G
     default: return false;
   }
@@ -641,7 +665,7 @@ cudaError_t launch_numeric_esc(cudaStream_t s, int sym_group, bool fp64, const N
   switch (sym_group) {
 #define SPG_G(I) \
   case I: return fp64 ? launch_num_esc_g<double, I>(s, a) : launch_num_esc_g<float, I>(s, a);
-    SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+    SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7)
 #undef SPG_G
     default: return cudaErrorInvalidValue;
   }

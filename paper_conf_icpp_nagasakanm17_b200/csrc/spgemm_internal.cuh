@@ -73,12 +73,12 @@ constexpr int kNumNumBounds = 13;
 constexpr int kNumCluster = 10;  // groups 10, 11, 12: clusters of 2, 4, 8 CTAs
 constexpr int kNumGlobal = 13;
 constexpr int kNumRange = 14;       // range rows (kernels_range.cu)
-// Batched expand-bucket-rank rows (kernels_esc.cu): numeric groups 15..21 hold the rows of
-// symbolic groups 2..8 whose n_prod_i <= ESC_PCT/100 * nnz_i (weak compression); a batch of them
+// Batched expand-bucket-rank rows (kernels_esc.cu): numeric groups 15..20 hold the rows of
+// symbolic groups 2..7 whose n_prod_i <= ESC_PCT/100 * nnz_i (weak compression); a batch of them
 // fits one CTA because the symbolic group bounds n_prod_i.
 constexpr int kNumEscBase = 15;
-constexpr int kEscSymLo = 2, kEscSymHi = 8;
-constexpr int kNumNumGroups = kNumEscBase + (kEscSymHi - kEscSymLo + 1);  // 22
+constexpr int kEscSymLo = 2, kEscSymHi = 7;
+constexpr int kNumNumGroups = kNumEscBase + (kEscSymHi - kEscSymLo + 1);  // 21
 
 // Range rows (kernels_range.cu): column span R_i <= kRangeMaxSpan and
 // R_i <= kRangeSpanPerProd * n_prod_i, n_prod_i in [range_min_np, kRangeMaxNprod] (one warp

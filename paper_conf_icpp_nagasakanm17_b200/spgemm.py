@@ -118,7 +118,7 @@ class Handle:
     def grouping(self, phase: int):
         """(n_prod int64[m], perm int32[m], offsets int64[ngroups+1]) of the last symbolic call."""
         m = self._A.m
-        ng = 13 if phase == 1 else 22  # groups incl. cluster, global, range and batched ESC (numeric)
+        ng = 13 if phase == 1 else 21  # groups incl. cluster, global, range and batched ESC (numeric)
         nprod = np.empty(m, dtype=np.int64)
         perm = np.empty(m, dtype=np.int32)
         off = np.zeros(ng + 1, dtype=np.int64)
