@@ -288,6 +288,33 @@ def _rmat_numpy(scale: int, edge_factor: int = 16, a: float = 0.45, b: float = 0
     return Csr(N, N, rpt, col, None, f"rmat{scale}")
 
 
+def aggregation_prolongator(n: int, agg: int = 2, smoothed: bool = True, seed: int = 0) -> Csr:
+    """AMG prolongator of the n x n 5-point grid (the Galerkin product R A P of
+    algebraic multigrid is a chained SpGEMM).  Aggregates are agg x agg blocks of grid points;
+    coarse point c = (x // agg) * ceil(n / agg) + y // agg.  Tentative prolongator: one entry per
+    fine point (its aggregate).  smoothed=True gives the STRUCTURE of the smoothed-aggregation
+    prolongator (I - w D^-1 A) P_tent — row i holds the aggregates of i and of its grid neighbours —
+    built combinatorially (no product is formed here); values are seeded U(0.5, 1.5)."""
+    nc = -(-n // agg)
+    idx = np.arange(n * n, dtype=np.int64)
+    x, y = idx // n, idx % n
+    R, C = [idx], [(x // agg) * nc + y // agg]
+    if smoothed:
+        for dx, dy in ((1, 0), (-1, 0), (0, 1), (0, -1)):
+            ok = (x + dx >= 0) & (x + dx < n) & (y + dy >= 0) & (y + dy < n)
+            R.append(idx[ok]); C.append(((x[ok] + dx) // agg) * nc + (y[ok] + dy) // agg)
+    Pm = from_coo(n * n, nc * nc, np.concatenate(R), np.concatenate(C), name=f"prolongator{n}")
+    return Pm.with_values("positive", seed)
+
+
+def transpose(M: Csr) -> Csr:
+    """CSR of M^T (a format conversion: the same entries, rows and columns swapped)."""
+    rows = np.repeat(np.arange(M.m, dtype=np.int64), np.diff(M.rpt))
+    T = from_coo(M.n, M.m, M.col.astype(np.int64), rows, M.val, dedup=False, name=M.name + "^T")
+    T.meta = dict(M.meta)
+    return T
+
+
 def random_sparse(m: int, n: int, density: float, seed: int, dup: bool = False,
                   unsorted: bool = False) -> Csr:
     """Small random pattern for brute-force pins; optional duplicate/unsorted columns."""

@@ -813,3 +813,50 @@ def test_graph_replay_new_structure_same_shape(spg):
             torch.cuda.synchronize()
             assert_parity(C.numpy() + (None,), ref, np.float32, what=f"call {it}")
             del C
+
+
+# ------------------------------------------------------------------ Galerkin product R A P (f3)
+
+def _galerkin_inputs(n):
+    A = synth.poisson2d(n)
+    P = synth.aggregation_prolongator(n, agg=2, smoothed=True, seed=3)
+    return A, P, synth.transpose(P)
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_galerkin_rap_chained(spg, dtype):
+    """AMG's R A P as two chained rectangular multiplies through the ABI, the
+    second reading the first's device output; both against the oracle."""
+    A, Pm, R = _galerkin_inputs(96)
+    AP_ref = oracle.spgemm(A.astype(dtype), Pm.astype(dtype), dtype)
+    AP_h = Csr(A.m, Pm.n, AP_ref[0], AP_ref[1], AP_ref[2].astype(np.float64))
+    RAP_ref = oracle.spgemm(R.astype(dtype), AP_h.astype(dtype), dtype)
+    with spg.Handle() as h:
+        AP = h.multiply(_dev(spg, A, dtype), _dev(spg, Pm, dtype))
+        torch.cuda.synchronize()
+        assert_parity(AP.numpy() + (None,), AP_ref, dtype, what="A P")
+        # the oracle's second product starts from its own A P; compare structure exactly and
+        # values within the tolerance of that product
+        RAP = h.multiply(_dev(spg, R, dtype), AP)
+        torch.cuda.synchronize()
+        assert_parity(RAP.numpy() + (None,), RAP_ref, dtype, what="R (A P)")
+        assert (RAP.m, RAP.n) == (Pm.n, Pm.n)
+
+
+def test_numeric_rerun_new_values(spg):
+    """Structure reuse: one symbolic phase, then numeric re-runs with new values
+    of A and B (same structures) into the same C buffers; every run against the oracle."""
+    A, Pm, _ = _galerkin_inputs(64)
+    with spg.Handle() as h:
+        dA, dP = _dev(spg, A, np.float64), _dev(spg, Pm, np.float64)
+        c_rpt, nnz, _ = h.symbolic(dA, dP)
+        c_col = torch.empty(nnz, dtype=torch.int32, device="cuda")
+        c_val = torch.empty(nnz, dtype=torch.float64, device="cuda")
+        for seed in range(3):
+            A2 = A.with_values("int", 10 + seed)
+            P2 = Pm.with_values("int", 20 + seed)
+            h.numeric(torch.from_numpy(A2.val).cuda(), torch.from_numpy(P2.val).cuda(), c_col, c_val)
+            torch.cuda.synchronize()
+            ref = oracle.spgemm(A2, P2, np.float64)
+            got = (c_rpt.cpu().numpy(), c_col.cpu().numpy(), c_val.cpu().numpy())
+            assert_parity(got + (None,), ref, np.float64, exact=True, what=f"re-run {seed}")

@@ -365,3 +365,35 @@ def test_parallel_oracle_identical(name, dtype):
         assert np.array_equal(x, y)
     assert np.array_equal(oracle.symbolic_omp(A, A), s[0])
     assert oracle.threads() >= 1 and oracle.cores() >= 1
+
+
+# ----------------------------------------------------------------- Galerkin product (chained, rectangular)
+
+def test_galerkin_rap_closed_form():
+    """PAPER.md:14, 302 (AMG's Galerkin product): with the tentative aggregation prolongator of 2x2
+    aggregates (one 1 per fine row) on the n x n 5-point Laplacian, R A P (R = P^T) sums A over
+    pairs of aggregates: an interior coarse row is again a 5-point stencil, 8 on the diagonal
+    (4 points x 4 minus their 8 internal links) and -2 to each edge neighbour (2 crossing links)."""
+    n = 8
+    A = synth.poisson2d(n)
+    P = synth.aggregation_prolongator(n, smoothed=False)
+    P = Csr(P.m, P.n, P.rpt, P.col, np.ones(P.nnz), P.name)
+    R = synth.transpose(P)
+    rpt, col, val, _ = oracle.spgemm(A, P, np.float64)
+    AP = Csr(A.m, P.n, rpt, col, val)
+    assert (AP.m, AP.n) == (64, 16)
+    rpt2, col2, val2, _ = oracle.spgemm(R, AP, np.float64)
+    nc = n // 2
+    for I in range(nc * nc):
+        cx, cy = I // nc, I % nc
+        row = dict(zip(col2[rpt2[I]:rpt2[I + 1]].tolist(), val2[rpt2[I]:rpt2[I + 1]].tolist()))
+        want = {I: 8.0}  # 4 diagonals of 4 minus 4 internal links counted both ways (A's diagonal is 4 everywhere)
+        for dx, dy in ((1, 0), (-1, 0), (0, 1), (0, -1)):
+            if 0 <= cx + dx < nc and 0 <= cy + dy < nc:
+                want[(cx + dx) * nc + cy + dy] = -2.0
+        assert row == want, (I, row, want)
+    # R A P of a symmetric A is symmetric
+    D = np.zeros((nc * nc, nc * nc))
+    for I in range(nc * nc):
+        D[I, col2[rpt2[I]:rpt2[I + 1]]] = val2[rpt2[I]:rpt2[I + 1]]
+    assert np.array_equal(D, D.T)

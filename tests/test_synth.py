@@ -87,3 +87,18 @@ def test_rmat_c_matches_numpy_twin(scale, seed):
     from synth.matrices import _rmat_numpy
     A, B = synth.rmat(scale, seed=seed), _rmat_numpy(scale, seed=seed)
     assert np.array_equal(A.rpt, B.rpt) and np.array_equal(A.col, B.col)
+
+
+def test_aggregation_prolongator_structure():
+    """Tentative: one entry per fine row (its 2x2 aggregate); smoothed: the aggregates of the row's
+    point and of its grid neighbours; transpose is an involution."""
+    n = 10
+    T = synth.aggregation_prolongator(n, smoothed=False)
+    assert (T.m, T.n) == (100, 25) and np.all(np.diff(T.rpt) == 1)
+    assert T.col[3 * n + 7] == (3 // 2) * 5 + 7 // 2
+    S = synth.aggregation_prolongator(n)
+    _check_csr(S)
+    i = 4 * n + 5  # (4, 5): its aggregate (2, 2) and the neighbours' (1|2, 2) and (2, 2|3)
+    assert S.col[S.rpt[i]:S.rpt[i + 1]].tolist() == sorted({2 * 5 + 2, 1 * 5 + 2, 2 * 5 + 3})
+    TT = synth.transpose(synth.transpose(S))
+    assert np.array_equal(TT.rpt, S.rpt) and np.array_equal(TT.col, S.col) and np.array_equal(TT.val, S.val)
