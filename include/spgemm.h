@@ -190,8 +190,13 @@ typedef enum {
                                        Off while the matching MIN_GROUP is forced */
     SPGEMM_OPT_ESC_PCT = 22,        /* compression bound of the ESC rows (default 200: n_prod_i <=
                                        2 nnz_i) */
-    SPGEMM_OPT_ESC_GROUPS = 23      /* bit g: rows of symbolic group g (2..8) may take the ESC kernels;
+    SPGEMM_OPT_ESC_GROUPS = 23,     /* bit g: rows of symbolic group g (2..7) may take the ESC kernels;
                                        -1 (default) = the library's rule */
+    SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
+                                       n_prod_i <= 32 run each phase as one thread-per-row launch
+                                       (register tables, no grouping, one host sync); otherwise,
+                                       or with 0, the grouped path.  spgemm_get_grouping then
+                                       returns SPGEMM_ERR_BAD_STATE */
 } spgemm_option_t;
 
 SPGEMM_API spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_t value);

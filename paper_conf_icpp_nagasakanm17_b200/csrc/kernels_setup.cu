@@ -519,6 +519,48 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_down(long long m, int64_
   }
 }
 
+// One-CTA inclusive scan of x[0..m) for small m (the small-matrix path): one launch instead of
+// three; chunks of 4096 staged through shared memory with coalesced loads and stores, a running
+// carry across chunks.
+constexpr int kSmallScanChunk = 4096;
+__global__ __launch_bounds__(1024) void k_scan_small(long long m, int64_t* __restrict__ x,
+                                                     long long* __restrict__ total_out) {
+  __shared__ long long tile[kSmallScanChunk];
+  __shared__ long long ws[33];
+  constexpr int PER = kSmallScanChunk / 1024;
+  long long carry = 0;
+  for (long long c = 0; c < m; c += kSmallScanChunk) {
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+      const long long i = c + e * 1024 + threadIdx.x;
+      tile[e * 1024 + threadIdx.x] = i < m ? x[i] : 0;
+    }
+    __syncthreads();
+    long long v[PER], s = 0;
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+      v[e] = tile[threadIdx.x * PER + e];
+      s += v[e];
+    }
+    long long tot;
+    long long run = carry + Grp<1024>::excl_scan(s, &tot, ws);
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+      run += v[e];
+      tile[threadIdx.x * PER + e] = run;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+      const long long i = c + e * 1024 + threadIdx.x;
+      if (i < m) x[i] = tile[e * 1024 + threadIdx.x];
+    }
+    carry += tot;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0 && total_out) *total_out = carry;
+}
+
 // ------------------------------------------------------------------ validation
 __global__ void k_validate(long long m, long long k, long long n, const int64_t* __restrict__ a_rpt,
                            const int32_t* __restrict__ a_col, const int64_t* __restrict__ b_rpt,
@@ -633,6 +675,12 @@ cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, c
                                   uint8_t* grp2, DevAcc* acc, Bounds b, EscSel esc, long long* tile_ws,
                                   int* nlaunch) {
   return scan_inclusive(s, m, c_rpt + 1, grp1, grp2, acc, b, esc, tile_ws, &acc->nnzc, nlaunch);
+}
+
+cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc) {
+  if (m <= 0) return cudaSuccess;
+  k_scan_small<<<1, 1024, 0, s>>>(m, c_rpt + 1, &acc->nnzc);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,

@@ -134,7 +134,167 @@ __global__ __launch_bounds__(128) void k_num_tiny(NumArgs a) {
     }
 }
 
+// Small matrices (m <= kSmallRows), whole phases in one launch each, a WARP per row and a lane
+// per product (rows with nnz(A_i) <= 32 and n_prod_i <= 32; a row above flags an overflow and the
+// host runs the general grouped path instead).  n_prod_i (Alg. 2) comes from the same pass.  The
+// row's loads take four dependent rounds whatever its shape (a_rpt; col_A, one per lane; the
+// rpt_B pairs; one B entry per lane), the products are ordered by a 32-lane bitonic network on
+// (column, value) pairs, equal columns are adjacent and summed (numeric, working precision,
+// PAPER.md:179), and each distinct column's position is the count of distinct columns below it
+// (PAPER.md:173's rank): no grouping, no shared memory, no sync 1.
+constexpr unsigned kFullW = 0xffffffffu;
+
+template <bool NUM, typename VT>
+__device__ __forceinline__ bool small_warp_row(const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
+                                               const VT* __restrict__ a_val, const int64_t* __restrict__ b_rpt,
+                                               const int32_t* __restrict__ b_col, const VT* __restrict__ b_val,
+                                               int row, int lane, int& key, VT& val, long long& np_out) {
+  const long long a0 = __ldg(a_rpt + row), a1 = __ldg(a_rpt + row + 1);
+  const int na = (int)(a1 - a0);
+  long long b0 = 0;
+  int len = 0;
+  VT av = VT(0);
+  if (lane < na) {
+    const int kk = __ldg(a_col + a0 + lane);
+    if (NUM) av = __ldg(a_val + a0 + lane);
+    b0 = __ldg(b_rpt + kk);
+    len = (int)(__ldg(b_rpt + kk + 1) - b0);
+  }
+  long long np = len;
+  for (long long j = a0 + 32 + lane; j < a1; j += 32) {  // rows longer than 32: n_prod only
+    const int k2 = __ldg(a_col + j);
+    np += __ldg(b_rpt + k2 + 1) - __ldg(b_rpt + k2);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) np += __shfl_xor_sync(kFullW, np, o);
+  np_out = np;
+  if (na > 32 || np > 32) return false;  // warp-uniform
+  int incl = len;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int y = __shfl_up_sync(kFullW, incl, d);
+    if (lane >= d) incl += y;
+  }
+  // product `lane` (Alg. 1 order) -> entry e = #entries whose inclusive prefix <= lane
+  int ent = 0;
+#pragma unroll
+  for (int st = 16; st > 0; st >>= 1)
+    if (__shfl_sync(kFullW, incl, ent + st - 1) <= lane) ent += st;
+  const int ex = __shfl_sync(kFullW, incl - len, ent);
+  const long long eb = __shfl_sync(kFullW, b0, ent);
+  const VT ea = NUM ? __shfl_sync(kFullW, av, ent) : VT(0);
+  key = INT_MAX;
+  val = VT(0);
+  if (lane < np) {
+    const long long q = eb + (lane - ex);
+    key = __ldg(b_col + q);
+    if (NUM) val = ea * __ldg(b_val + q);
+  }
+  // bitonic sort of (key, val) over the 32 lanes, ascending
+#pragma unroll
+  for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      const int ok = __shfl_xor_sync(kFullW, key, j);
+      const VT ov = NUM ? __shfl_xor_sync(kFullW, val, j) : VT(0);
+      const bool up = (lane & k) == 0;           // this pair sorts ascending
+      const bool lower = (lane & j) == 0;        // this lane keeps the smaller key
+      const bool take = up == lower ? ok < key : ok > key;
+      if (take) {
+        key = ok;
+        if (NUM) val = ov;
+      }
+    }
+  }
+  return true;
+}
+
+__global__ __launch_bounds__(128) void k_small_sym(long long m, long long k, const int64_t* __restrict__ a_rpt,
+                                                   const int32_t* __restrict__ a_col, const int64_t* __restrict__ b_rpt,
+                                                   const int32_t* __restrict__ b_col, int64_t* __restrict__ c_cnt,
+                                                   int64_t* __restrict__ nprod, DevAcc* acc) {
+  const long long row = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (row == 0 && lane == 0) {  // what the host needs besides nnz(C): nnz(A), nnz(B)
+    acc->ends[0] = a_rpt[0]; acc->ends[1] = a_rpt[m]; acc->ends[2] = b_rpt[0]; acc->ends[3] = b_rpt[k];
+  }
+  if (row >= m) return;  // warp-uniform
+  int key;
+  int dummy;
+  long long np;
+  const bool fast = small_warp_row<false, int>(a_rpt, a_col, nullptr, b_rpt, b_col, nullptr, (int)row, lane, key,
+                                               dummy, np);
+  int n = 0;
+  if (fast) {
+    const int prev = __shfl_up_sync(kFullW, key, 1);
+    n = __popc(__ballot_sync(kFullW, key != INT_MAX && (lane == 0 || prev != key)));
+  } else if (np > 0 && lane == 0) {
+    atomicAdd(&acc->small_overflow, 1);
+  }
+  if (lane == 0) {
+    nprod[row] = np;
+    c_cnt[row] = n;
+    atomicAdd(&acc->total_nprod, (unsigned long long)np);
+    atomicMax(&acc->max_nprod, (unsigned long long)np);
+  }
+}
+
+template <typename VT>
+__global__ __launch_bounds__(128) void k_small_num(NumArgs a, long long m) {
+  const long long row = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (row >= m) return;  // warp-uniform
+  int key;
+  VT val;
+  long long np;
+  const bool fast = small_warp_row<true, VT>(a.a_rpt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt, a.b_col,
+                                             static_cast<const VT*>(a.b_val), (int)row, lane, key, val, np);
+  const long long c0 = a.c_rpt[row];
+  const int cn = (int)(a.c_rpt[row + 1] - c0);
+  if (!fast) {
+    if (np > 0 && lane == 0) atomicOr(a.err_flags, 2);
+    return;
+  }
+  const int prev = __shfl_up_sync(kFullW, key, 1);
+  const bool head = key != INT_MAX && (lane == 0 || prev != key);
+  // sum each run of equal keys into its head: segmented suffix sums over the lanes
+  VT run = val;
+  int seg = key;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const VT y = __shfl_down_sync(kFullW, run, d);
+    const int ky = __shfl_down_sync(kFullW, seg, d);
+    if (lane + d < 32 && ky == key) run += y;
+  }
+  const unsigned hm = __ballot_sync(kFullW, head);
+  if (__popc(hm) != cn) {
+    if (lane == 0) atomicOr(a.err_flags, 2);
+    return;
+  }
+  if (head) {
+    const int pos = __popc(hm & ((1u << lane) - 1u));
+    a.c_col[c0 + pos] = key;
+    static_cast<VT*>(a.c_val)[c0 + pos] = run;
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_small_symbolic(cudaStream_t s, long long m, long long k, const int64_t* a_rpt, const int32_t* a_col,
+                                  const int64_t* b_rpt, const int32_t* b_col, int64_t* c_cnt, int64_t* nprod,
+                                  DevAcc* acc) {
+  if (m <= 0) return cudaSuccess;
+  k_small_sym<<<(unsigned)((m * 32 + 127) / 128), 128, 0, s>>>(m, k, a_rpt, a_col, b_rpt, b_col, c_cnt, nprod, acc);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_small_numeric(cudaStream_t s, bool fp64, const NumArgs& a, long long m) {
+  if (m <= 0) return cudaSuccess;
+  const unsigned grid = (unsigned)((m * 32 + 127) / 128);
+  if (fp64) k_small_num<double><<<grid, 128, 0, s>>>(a, m);
+  else k_small_num<float><<<grid, 128, 0, s>>>(a, m);
+  return cudaGetLastError();
+}
 
 // Groups served (capacity = the group's bound): symbolic 0 (n_prod <= 16), 1 (<= 32); numeric 0
 // (nnz <= 8), 1 (<= 16).

@@ -95,6 +95,8 @@ struct spgemm_ctx {
   // vs 4.5, group 7 (4096) 3.6 vs 4.6
   long long rank_l1_pct = 500, rank_l1_pct_sym = 150;
   int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
+  int small_opt = 1;     // small matrices (m <= kSmallRows): one-launch phases, no grouping (kernels_tiny.cu)
+  bool small = false;    // the last symbolic call took the small-matrix path
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
   // 26.5 ms vs 21.7 ms with the per-group hash / rank-count kernels), bit 2 numeric ESC
   int batch = 2;
@@ -120,6 +122,7 @@ struct spgemm_ctx {
       rbits, bbits;
   bool range_num = false;  // numeric range rows on for the last symbolic call (bitmap allocated, B sorted)
   GraphCache gsym, gnum;  // captured segments (see run_graph)
+  GraphCache gsmall;      // small-matrix symbolic segment
   int use_graphs = 1;
   bool perm2_ready = false;
   bool group_sums_done = false;  // per-group n_prod/nnz sums (computed on demand by get_stats)
@@ -496,6 +499,7 @@ spgemm_status_t spgemm_destroy(spgemm_handle_t h) {
     }
     if (h->gsym.exec) cudaGraphExecDestroy(h->gsym.exec);
     if (h->gnum.exec) cudaGraphExecDestroy(h->gnum.exec);
+    if (h->gsmall.exec) cudaGraphExecDestroy(h->gsmall.exec);
     for (int i = 0; i < kNumStreams; ++i) {
       if (h->gs[i]) cudaStreamDestroy(h->gs[i]);
       if (h->join_ev[i]) cudaEventDestroy(h->join_ev[i]);
@@ -579,6 +583,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       if (v < 0 || v > (1LL << 40)) return fail(h, SPGEMM_ERR_INVALID_ARG, "ESC_PCT out of range");
       h->esc_pct = v; break;
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
+    case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -611,10 +616,14 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   h->stats.n_num_groups = kNumNumGroups;
   long long launches = 0;
 
-  CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));
   ALLOC(h->acc, sizeof(DevAcc));
-  CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
   DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+  const bool small_try = h->small_opt && m > 0 && m <= kSmallRows && h->sym_min_group < 0 && h->num_min_group < 0 &&
+                         h->tiny >= 1 && !h->validate;
+  if (!small_try) {
+    CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));
+    CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
+  }
   if (m == 0) {
     CK(cudaStreamSynchronize(h->stream));
     h->nnzc = 0; h->nnza = 0; h->nnzb = 0;
@@ -645,6 +654,60 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
     CK(cudaStreamSynchronize(h->stream));
     if (h->hacc->err_flags & 1)
       return fail(h, SPGEMM_ERR_INVALID_INPUT, "input validation failed (rpt not monotone or col out of range)");
+  }
+  // Small matrices: thread-per-row symbolic count with n_prod (Alg. 2) in the same pass and a
+  // register table (rows with n_prod_i <= kSmallCap), then the rpt scan and one sync; rows above
+  // the cap send the call down the general grouped path below.
+  h->small = false;
+  if (small_try) {
+    // zero the counters, count, scan, copy the counters back: one captured segment (one graph
+    // launch per call once the pointers repeat)
+    const std::vector<long long> topo = {3, m, k, n, (long long)group_events(h)};
+    const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
+                                         (long long)c_rpt, (long long)h->acc.p, (long long)h->nprod.p,
+                                         (long long)h->hacc};
+    auto enqueue = [&]() -> spgemm_status_t {
+      CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));
+      CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
+      CK(launch_small_symbolic(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, c_rpt + 1,
+                               static_cast<int64_t*>(h->nprod.p), dacc));
+      CK(launch_scan_small(h->stream, m, c_rpt, dacc));
+      CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
+      return SPGEMM_OK;
+    };
+    const spgemm_status_t ss = run_graph(h, h->gsmall, topo, ptrs, enqueue);
+    if (ss != SPGEMM_OK) return ss;
+    const int nl = 2;
+    CK(cudaStreamSynchronize(h->stream));  // the only host sync of the small path: nnz(C)
+    if (h->hacc->small_overflow == 0) {
+      h->snap1 = h->snap2 = *h->hacc;
+      h->small = true;
+      h->nnza = h->hacc->ends[1] - h->hacc->ends[0];
+      h->nnzb = h->hacc->ends[3] - h->hacc->ends[2];
+      h->nnzc = h->snap2.nnzc;
+      *c_nnz = h->nnzc;
+      if (nprod_out) *nprod_out = (int64_t)h->snap1.total_nprod;
+      if (h->timing) {
+        CK(cudaEventRecord(h->ev[3], h->stream));
+        h->gtimed_phases = false;
+      }
+      spgemm_stats_t& st = h->stats;
+      st.nnz_a = h->nnza; st.nnz_b = h->nnzb; st.nnz_c = h->nnzc;
+      st.nprod = (int64_t)h->snap1.total_nprod;
+      st.max_row_nprod = (int64_t)h->snap1.max_nprod;
+      st.sym_rows[0] = st.num_rows[0] = m;
+      st.sym_nprod[0] = st.num_nprod[0] = st.nprod;
+      st.sym_nnza[0] = st.num_nnza[0] = h->nnza;
+      st.num_nnzc[0] = h->nnzc;
+      h->gkind[0][0] = SPGEMM_KERNEL_TINY;
+      h->group_sums_done = true;
+      st.kernel_launches_symbolic = launches + 1 + nl;
+      h->state = 1;
+      CK(leave(h));
+      return SPGEMM_OK;
+    }
+    CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));  // general path from scratch
+    CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
   }
   // (1)+(2): n_prod per row (Alg. 2), column spans, group ids / histogram
   {
@@ -744,7 +807,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->range_hash, (long long)group_events(h), h->range_warp, h->range_min_np,
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
                                  (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym,
-                                 (long long)h->sym_min_group, (long long)h->batch, h->esc_pct, h->esc_mask};
+                                 (long long)h->sym_min_group, (long long)h->batch, h->esc_pct, h->esc_mask,
+                                 (long long)h->small_opt};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -921,7 +985,16 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
   memset(h->gkind[1], 0, sizeof h->gkind[1]);
   h->numeric_done = true;
   if (h->timing) CK(cudaEventRecord(h->ev[4], h->stream));
-  if (h->m > 0 && h->nnzc > 0) {
+  if (h->small && h->nnzc > 0) {  // small-matrix path: one thread-per-row launch (kernels_tiny.cu)
+    NumArgs na{};
+    na.a_rpt = h->a_rpt; na.a_col = h->a_col; na.a_val = a_val;
+    na.b_rpt = h->b_rpt; na.b_col = h->b_col; na.b_val = b_val;
+    na.c_rpt = h->c_rpt; na.c_col = c_col; na.c_val = c_val;
+    na.err_flags = &static_cast<DevAcc*>(h->acc.p)->err_flags;
+    CK(launch_small_numeric(h->stream, dt == SPGEMM_F64, na, h->m));
+    h->gkind[1][0] = SPGEMM_KERNEL_TINY;
+    h->stats.kernel_launches_numeric = 1;
+  } else if (h->m > 0 && h->nnzc > 0) {
     spgemm_status_t s = ensure_perm2(h);
     if (s != SPGEMM_OK) return s;
     const bool fp64 = dt == SPGEMM_F64;
@@ -1201,6 +1274,8 @@ spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t* out) {
 spgemm_status_t spgemm_get_grouping(spgemm_handle_t h, int phase, int64_t* nprod, int32_t* perm, int64_t* offsets) {
   if (!h || (phase != 1 && phase != 2)) return SPGEMM_ERR_INVALID_ARG;
   if (h->state != 1) return fail(h, SPGEMM_ERR_BAD_STATE, "no symbolic result");
+  if (h->small)
+    return fail(h, SPGEMM_ERR_BAD_STATE, "the small-matrix path builds no grouping (set SPGEMM_OPT_SMALL 0)");
   DeviceGuard dg(h->device);
   CK(enter(h));
   if (h->m == 0) {

@@ -137,7 +137,14 @@ struct DevAcc {  // zeroed at the start of spgemm_symbolic, copied to pinned hos
   int row_counter[4];  // numeric cluster groups: dynamic row counters (zeroed per numeric call)
   int defer_count[2];  // step (1): deferred long rows of B (0) and A (1)
   int bbits_wmax;      // range rows: max words of a B-row bitmap (k_brow_bits)
+  int small_overflow;  // small-matrix path: rows with n_prod_i > kSmallCap (-> general path)
+  long long ends[4];   // small-matrix path: a_rpt[0], a_rpt[m], b_rpt[0], b_rpt[k]
 };
+
+// Small matrices (m <= kSmallRows): one-launch symbolic and numeric phases, thread per row with a
+// register table of kSmallCap slots (kernels_tiny.cu), no grouping and no sync 1.
+constexpr long long kSmallRows = 65536;
+constexpr int kSmallCap = 32;
 
 struct Bounds {  // group bounds passed by value
   long long upper[kMaxGroups];
@@ -798,6 +805,7 @@ cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, c
                                   uint8_t* grp2, DevAcc* acc, Bounds b, EscSel esc,
                                   long long* tile_ws, int* nlaunch);
 size_t scan_workspace_bytes(long long m);
+cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc);
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
                             const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int* err);
 cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,
@@ -814,6 +822,10 @@ cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a)
 int rankcnt_smem_bytes(int group, int l1_words);
 cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid);
 cudaError_t launch_symbolic_tiny(cudaStream_t s, int group, const SymArgs& a);
+cudaError_t launch_small_symbolic(cudaStream_t s, long long m, long long k, const int64_t* a_rpt, const int32_t* a_col,
+                                  const int64_t* b_rpt, const int32_t* b_col, int64_t* c_cnt, int64_t* nprod,
+                                  DevAcc* acc);
+cudaError_t launch_small_numeric(cudaStream_t s, bool fp64, const NumArgs& a, long long m);
 cudaError_t launch_numeric_tiny(cudaStream_t s, int group, bool fp64, const NumArgs& a);
 int rankbig_smem_bytes(bool fp64, int l1_words);
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
