@@ -192,6 +192,11 @@ typedef enum {
                                        2 nnz_i) */
     SPGEMM_OPT_ESC_GROUPS = 23,     /* bit g: rows of symbolic group g (2..7) may take the ESC kernels;
                                        -1 (default) = the library's rule */
+    SPGEMM_OPT_WSORT = 25,          /* warp-per-row register sort, bit mask: 1 =
+                                       symbolic groups 2-5 (n_prod_i <= 1024) count distinct columns of
+                                       a bitonic-sorted register row; 2 = numeric rows of those groups
+                                       with 100 * n_prod_i <= ESC_PCT * nnz_i.  Default 0 (measured
+                                       slower than the hash / ESC kernels: ablation) */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,
@@ -235,7 +240,8 @@ typedef enum {
     SPGEMM_KERNEL_RANK_BIG = 6, /* rank-indexed, level 2 in global memory, values reduced into C */
     SPGEMM_KERNEL_TINY = 7,     /* thread per row, sorted register table (kernels_tiny.cu)       */
     SPGEMM_KERNEL_BATCH = 8,    /* batched rows per CTA, paper hash in shared memory (symbolic)   */
-    SPGEMM_KERNEL_ESC = 9       /* batched expand-bucket-rank-compress rows (kernels_esc.cu)      */
+    SPGEMM_KERNEL_ESC = 9,      /* batched expand-bucket-rank-compress rows (kernels_esc.cu)      */
+    SPGEMM_KERNEL_WSORT = 10    /* warp per row, bitonic-sorted register row (kernels_wsort.cu)   */
 } spgemm_kernel_t;
 
 SPGEMM_API spgemm_status_t spgemm_get_stats(spgemm_handle_t h, spgemm_stats_t *out /* host */);

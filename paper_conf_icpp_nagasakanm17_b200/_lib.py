@@ -27,11 +27,11 @@ OPTIONS = {
     "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8, "range_hash": 9,
     "cluster": 10, "cluster_fill_limit": 11, "flat": 12, "graphs": 13, "range_warp": 14,
     "range_min_nprod": 15, "bitmap_rank": 16, "rank_acc": 17, "tiny": 18, "rank_l1_pct": 19, "rank_l1_pct_sym": 20,
-    "batch": 21, "esc_pct": 22, "esc_groups": 23, "small": 24,
+    "batch": 21, "esc_pct": 22, "esc_groups": 23, "small": 24, "wsort": 25,
 }
 
 # spgemm_kernel_t (include/spgemm.h): kernel family that ran each group
-KERNELS = {0: "none", 1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big", 7: "tiny", 8: "batch", 9: "esc"}
+KERNELS = {0: "none", 1: "hash", 2: "rank", 3: "range", 4: "cluster", 5: "global", 6: "rank_big", 7: "tiny", 8: "batch", 9: "esc", 10: "wsort"}
 
 # Group ids of the range-row kernels (spgemm_internal.cuh kSymRange / kNumRange).
 SYM_RANGE_GROUP = 12

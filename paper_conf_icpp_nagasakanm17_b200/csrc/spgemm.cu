@@ -96,6 +96,11 @@ struct spgemm_ctx {
   long long rank_l1_pct = 500, rank_l1_pct_sym = 150;
   int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
   int small_opt = 1;     // small matrices (m <= kSmallRows): one-launch phases, no grouping (kernels_tiny.cu)
+  // warp-per-row register sort (kernels_wsort.cu): bit 1 symbolic, bit 2 numeric.  Off by default:
+  // measured 2.5-9x slower than the hash / ESC kernels on every graph config (R-MAT s16-s22, webbase,
+  // Economics, Circuit; scripts/ab.py): the unrolled networks' register footprint (up to 240 per
+  // thread) leaves 8-16 warps per SM and the shuffle stages serialise
+  int wsort = 0;
   bool small = false;    // the last symbolic call took the small-matrix path
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
   // 26.5 ms vs 21.7 ms with the per-group hash / rank-count kernels), bit 2 numeric ESC
@@ -382,6 +387,8 @@ bool flat_of(spgemm_handle_t h) {
 unsigned esc_auto_mask(spgemm_handle_t h) {
   const long long W = h->n / 1024 + 1;
   unsigned m = 0;
+  if (h->wsort & 2)  // warp-sorted rows (kernels_wsort.cu): groups 2..wsort_max_group() on any matrix
+    for (int g = kEscSymLo; g <= wsort_max_group(); ++g) m |= 1u << g;
   for (int g = kEscSymLo; g <= kEscSymHi; ++g)
     if (100 * W >= h->esc_w_pct * kSymGroups[g].upper && W > 1024) m |= 1u << g;
   return m;
@@ -584,6 +591,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->esc_pct = v; break;
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
+    case SPGEMM_OPT_WSORT:
+      if (v < 0 || v > 3) return fail(h, SPGEMM_ERR_INVALID_ARG, "WSORT must be 0..3");
+      h->wsort = (int)v; break;
     case SPGEMM_OPT_LONG_ROW:
       if (v < -1 || v > (1 << 30)) return fail(h, SPGEMM_ERR_INVALID_ARG, "LONG_ROW out of range");
       h->long_len = (int)v; break;
@@ -772,6 +782,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   sa.err_flags = &dacc->err_flags;
   // batched paper-hash symbolic kernels for groups 2-9 (kernels_esc.cu)
   auto batch_sym_on = [&](int g) { return (h->batch & 1) && h->sym_min_group < 0 && g >= 2 && g <= 9; };
+  auto wsort_sym_on = [&](int g) { return (h->wsort & 1) && h->sym_min_group < 0 && g >= 2 && g <= wsort_max_group(); };
   // rank-count kernels for the CTA-per-row groups (kernels_rankacc.cu; needs the column spans)
   auto rank_cnt_on = [&](int g) {
     return h->rank_acc && h->rlohi.p != nullptr && h->sym_min_group < 0 && g >= 5 && g <= 9 &&
@@ -808,7 +819,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
                                  (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym,
                                  (long long)h->sym_min_group, (long long)h->batch, h->esc_pct, h->esc_mask,
-                                 (long long)h->small_opt};
+                                 (long long)h->small_opt, (long long)h->wsort};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -837,10 +848,11 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       ga.nrows = rows;
       const bool tiny_g = h->tiny >= 2 && h->sym_min_group < 0 && g <= 1;  // measured slower than the hash
       if (tiny_g) CK(launch_symbolic_tiny(s, g, ga));
+      else if (wsort_sym_on(g)) CK(launch_symbolic_wsort(s, g, ga));
       else if (batch_sym_on(g)) CK(launch_symbolic_batch(s, g, ga));
       else if (rank_cnt_on(g)) CK(launch_symbolic_rankcnt(s, g, ga));
       else CK(launch_symbolic_group(s, g, ga, h->num_sms));
-      h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : batch_sym_on(g) ? SPGEMM_KERNEL_BATCH
+      h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : wsort_sym_on(g) ? SPGEMM_KERNEL_WSORT : batch_sym_on(g) ? SPGEMM_KERNEL_BATCH
                      : rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
       ++launches;
       if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
@@ -1073,7 +1085,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
                                    (long long)h->num_min_group, (long long)big_rank, (long long)h->snap2.max_nnz,
-                                   na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words};
+                                   na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words, (long long)h->wsort};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
                                          (long long)h->c_rpt, (long long)h->a_rpt, (long long)h->a_col,
@@ -1093,9 +1105,15 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
         NumArgs ga = na;
         ga.rows = perm2 + off2.off[g];
         ga.nrows = rows;
-        if (g >= kNumEscBase) {  // batched expand-bucket-rank rows (kernels_esc.cu)
-          h->gkind[1][g] = SPGEMM_KERNEL_ESC;
-          CK(launch_numeric_esc(st, g - kNumEscBase + kEscSymLo, fp64, ga));
+        if (g >= kNumEscBase) {  // weakly compressing rows grouped by n_prod: warp-sorted or ESC batches
+          const int sg = g - kNumEscBase + kEscSymLo;
+          if ((h->wsort & 2) && sg <= wsort_max_group()) {
+            h->gkind[1][g] = SPGEMM_KERNEL_WSORT;
+            CK(launch_numeric_wsort(st, sg, fp64, ga));
+          } else {
+            h->gkind[1][g] = SPGEMM_KERNEL_ESC;
+            CK(launch_numeric_esc(st, sg, fp64, ga));
+          }
         } else if (g == kNumGlobal) {
           h->gkind[1][g] = SPGEMM_KERNEL_GLOBAL;
           CK(launch_numeric_global(st, fp64, ga, glob_grid));

@@ -844,6 +844,9 @@ int cluster_capacity_sym();
 cudaError_t launch_symbolic_batch(cudaStream_t s, int group, const SymArgs& a);
 cudaError_t launch_numeric_esc(cudaStream_t s, int sym_group, bool fp64, const NumArgs& a);
 bool numeric_esc_supported(int sym_group, bool fp64);
+int wsort_max_group();
+cudaError_t launch_symbolic_wsort(cudaStream_t s, int sym_group, const SymArgs& a);
+cudaError_t launch_numeric_wsort(cudaStream_t s, int sym_group, bool fp64, const NumArgs& a);
 int cluster_capacity_num();
 
 }  // namespace spg

@@ -860,3 +860,17 @@ def test_numeric_rerun_new_values(spg):
             ref = oracle.spgemm(A2, P2, np.float64)
             got = (c_rpt.cpu().numpy(), c_col.cpu().numpy(), c_val.cpu().numpy())
             assert_parity(got + (None,), ref, np.float64, exact=True, what=f"re-run {seed}")
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+@pytest.mark.parametrize("name", ["rmat14", "webbase_small", "mixed:circuit"])
+def test_warp_sorted_rows(spg, name, dtype):
+    """WSORT ablation (kernels_wsort.cu): symbolic groups 2-5 count the distinct columns of a
+    bitonic-sorted register row; numeric rows of those groups are sorted, summed and compacted in
+    registers / warp-private shared memory."""
+    A = _mixed_small() if name == "webbase_small" else (
+        synth.rmat(14).with_values("uniform", 9) if name == "rmat14" else synth.config(name))
+    got = check(spg, A, A, dtype, opts={"wsort": 3}, what=f"{name} wsort")
+    st = got[3]
+    assert any(st["sym_kernel"][g] == 10 for g in range(2, 6) if st["sym_rows"][g]), st["sym_kernel"]
+    assert any(st["num_kernel"][g] == 10 for g in range(15, 19) if st["num_rows"][g]), st["num_kernel"]
