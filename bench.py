@@ -392,6 +392,23 @@ def run_ours(args):
                            "no other buffers"}
         del C
         hp.close()
+        # allocation of C (reading R18): warm (caching allocator) and cold (the
+        # cache emptied first: cudaMalloc of nnz(C) entries)
+        nnz_c = h.nnz_c
+        def alloc_ms():
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            cc = torch.empty(nnz_c, dtype=torch.int32, device=dev)
+            cv = torch.empty(nnz_c, dtype=tdt, device=dev)
+            e1.record()
+            torch.cuda.synchronize()
+            del cc, cv
+            return e0.elapsed_time(e1)
+        alloc_ms()
+        warm = statistics.median(alloc_ms() for _ in range(5))
+        torch.cuda.empty_cache()
+        cold = alloc_ms()
+        peak_mem["c_alloc_ms"] = {"warm": warm, "cold": cold, "bytes": int(nnz_c * (4 + vbytes))}
         flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
     # end to end through the public API: pinned host A -> device, (broadcast, split,) multiply,
