@@ -323,7 +323,7 @@ __device__ __forceinline__ int esc_scan_counts(int* c, int* ws, int (&vals)[N]) 
 }
 
 template <typename VT, int TPR, int KP, int MC, int R, int BM, bool REFINE>
-__global__ __launch_bounds__(TPR, (1024 / TPR)) void k_num_esc(NumArgs a) {
+__global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(NumArgs a) {
   constexpr int kEscBm = BM;
   using S = NumEscSmem<VT, TPR, KP, MC, R, BM, REFINE>;
   constexpr int CAP = S::CAP;
@@ -561,11 +561,23 @@ struct EscCfg {
 constexpr EscCfg kEscSym[] = {{0, 0, 0}, {0, 0, 0}, {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
                               {256, 8, 2}, {256, 8, 2}, {512, 8, 2}, {1024, 8, 2}, {1024, 16, 1}};
 #ifndef SPG_ESC_SMALL_TPR
-#define SPG_ESC_SMALL_TPR 256
+#define SPG_ESC_SMALL_TPR 128
 #endif
 constexpr int kEscSmallTpr = SPG_ESC_SMALL_TPR;
-constexpr EscCfg kEscNum32[] = {{0, 0, 0},  {0, 0, 0},  {kEscSmallTpr, 8, 2},  {kEscSmallTpr, 8, 2},  {kEscSmallTpr, 8, 2},
-                                {kEscSmallTpr, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
+#ifndef SPG_ESC_KP
+#define SPG_ESC_KP 8
+#endif
+constexpr int kEscKp = SPG_ESC_KP;  // products per thread (fp32); CAP = TPR * KP >= the group bound
+constexpr EscCfg kEscNum32[] = {{0, 0, 0},
+                                {0, 0, 0},
+                                {kEscSmallTpr, kEscKp, 2},
+                                {kEscSmallTpr, kEscKp, 2},
+                                {kEscSmallTpr, kEscKp, 2},
+                                {kEscSmallTpr * 8 / kEscKp >= 128 ? kEscSmallTpr * 8 / kEscKp : 128, kEscKp, 2},
+                                {256 * 8 / kEscKp, kEscKp, 2},
+                                {512 * 8 / kEscKp, kEscKp, 2},
+                                {1024, 8, 2},
+                                {1024, 16, 1}};
 constexpr EscCfg kEscNum64[] = {{0, 0, 0},  {0, 0, 0},  {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
                                 {256, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
 template <typename VT>
