@@ -322,7 +322,7 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
 }
 
 template <typename VT>
-constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 4 + (int)sizeof(BlockFlat<VT, 1024>); }
+constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 4 + (int)sizeof(BlockFlat<VT, 1024, 2048>); }
 
 // 40 registers (1536 threads per SM) for fp32 / symbolic; fp64 values need 64 (no spills)
 // (KP > 8 products per thread: 1280 threads, ~48 registers)
@@ -438,7 +438,7 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
   const int l1p = rankbig_l1pad_h(a.l1_words);
   unsigned* l1 = reinterpret_cast<unsigned*>(smem_raw);
   unsigned* p1 = l1 + l1p;
-  BlockFlat<VT, TPR>* bf = reinterpret_cast<BlockFlat<VT, TPR>*>(p1 + l1p);
+  BlockFlat<VT, TPR, 2048>* bf = reinterpret_cast<BlockFlat<VT, TPR, 2048>*>(p1 + l1p);
   unsigned* fine = reinterpret_cast<unsigned*>(static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride);
   unsigned* pre2 = fine + a.slab_T;
   const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val);

@@ -132,7 +132,7 @@ __global__ __launch_bounds__(BS) void k_sym_smem(SymArgs a) {
   __shared__ long long ws[33];
   __shared__ int s_cnt, s_abort, s_lcnt;
   __shared__ int s_list[TPR > 32 ? kLongChunk : 1];
-  using BF = BlockFlat<int, flat_chunk_of<TPR>()>;
+  using BF = BlockFlat<int, flat_chunk_of<TPR>(), (TPR > 32 ? 4 * flat_chunk_of<TPR>() : 0)>;
   __shared__ std::conditional_t<(TPR > 32), BF, int> s_bf_store;  // only CTA groups need it
   constexpr int RPB = BS / TPR;
   static_assert(BS % TPR == 0 && (TPR <= 32 || TPR == BS), "row group must be sub-warp or the CTA");

@@ -388,12 +388,17 @@ template <int TPR>
 struct Grp;  // row-group collectives (defined below)
 // N entries per chunk: kFlatChunk by default; the CTA-per-row group kernels use one chunk of TPR
 // entries (up to 1024) so that a row of <= TPR A non-zeros costs a single metadata round trip.
-template <typename VT, int N = kFlatChunk>
+// NB > 0: a block-start table — for each 32-product block of the chunk, the first A entry holding
+// one of its products — so a product finds its entry with one lookup and a short forward walk
+// instead of a binary search over the chunk (chunks of up to 32 * NB products; larger ones search).
+template <typename VT, int N = kFlatChunk, int NB = 0>
 struct BlockFlat {
   static constexpr int kN = N;
+  static constexpr int kNB = NB;
   long long b0[N];
   int incl[N];
   VT av[N];
+  int bstart[NB > 0 ? NB : 1];
 };
 template <int TPR>
 constexpr int flat_chunk_of() { return TPR < 1024 ? TPR : 1024; }
@@ -425,8 +430,11 @@ __device__ __forceinline__ void for_each_product_block(const int64_t* __restrict
     long long tot;
     const long long ex = Grp<TPR>::excl_scan(t < cn ? len : 0, &tot, ws);  // block scan
     if (t < cn) sh->incl[t] = (int)(ex + len);
+    const int P = (int)tot;  // CTA-uniform
+    const bool table = BF::kNB > 0 && P <= 32 * BF::kNB;
+    if (table && t < cn)  // 32-product blocks whose first product lies in this entry
+      for (int k = (int)((ex + 31) >> 5); k < (int)((ex + len + 31) >> 5); ++k) sh->bstart[k] = t;
     __syncthreads();
-    const int P = (int)tot;
     // kU products per thread per round: all kU gathers are issued before any table update (B rows
     // of graph shapes are short and scattered: each gather is an L2/HBM round trip)
     constexpr int kU = 4;
@@ -440,10 +448,17 @@ __device__ __forceinline__ void for_each_product_block(const int64_t* __restrict
         const int p = p0 + u * tpr;
         es[u] = -1;
         if (p < P) {
-          int lo = 0, hi = cn - 1;  // first e with incl[e] > p
-          while (lo < hi) {
-            const int mid = (lo + hi) >> 1;
-            if (sh->incl[mid] <= p) lo = mid + 1; else hi = mid;
+          int lo;  // first e with incl[e] > p
+          if (table) {
+            lo = sh->bstart[p >> 5];
+            while (sh->incl[lo] <= p) ++lo;
+          } else {
+            lo = 0;
+            int hi = cn - 1;
+            while (lo < hi) {
+              const int mid = (lo + hi) >> 1;
+              if (sh->incl[mid] <= p) lo = mid + 1; else hi = mid;
+            }
           }
           es[u] = lo;
           const int start = lo ? sh->incl[lo - 1] : 0;
