@@ -210,6 +210,18 @@ cudaError_t launch_sym(cudaStream_t s, const SymArgs& a) {
   return cudaGetLastError();
 }
 
+// Table slots of group I's hash kernel: kSymTableFactor x the Table-I size (load <= 1/(2 factor))
+// where the CTA's tables stay within 64 KB; the optimistic group keeps its fill-limited table.
+#ifndef SPG_SYM_TF
+#define SPG_SYM_TF 1
+#endif
+constexpr int kSymTableFactor = SPG_SYM_TF;
+template <int I>
+constexpr int sym_table() {
+  constexpr int T = kSymGroups[I].T, RPB = kSymGroups[I].BS / kSymGroups[I].TPR;
+  return (I != kSymOptimistic && RPB * T * kSymTableFactor * 4 <= 64 * 1024) ? T * kSymTableFactor : T;
+}
+
 }  // namespace
 
 cudaError_t launch_symbolic_group(cudaStream_t s, int group, const SymArgs& a, int /*num_sms*/) {
@@ -217,7 +229,7 @@ cudaError_t launch_symbolic_group(cudaStream_t s, int group, const SymArgs& a, i
   switch (group) {
 #define SPG_G(I)                                                                              \
   case I:                                                                                     \
-    return launch_sym<kSymGroups[I].T, kSymGroups[I].TPR, kSymGroups[I].BS, (I == kSymOptimistic)>(s, a);
+    return launch_sym<sym_table<I>(), kSymGroups[I].TPR, kSymGroups[I].BS, (I == kSymOptimistic)>(s, a);
     SPG_G(0) SPG_G(1) SPG_G(2) SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9) SPG_G(10)
 #undef SPG_G
     default: return cudaErrorInvalidValue;

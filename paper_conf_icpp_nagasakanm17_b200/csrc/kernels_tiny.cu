@@ -151,6 +151,8 @@ __device__ __forceinline__ bool small_warp_row(const int64_t* __restrict__ a_rpt
                                                int row, int lane, int& key, VT& val, long long& np_out) {
   const long long a0 = __ldg(a_rpt + row), a1 = __ldg(a_rpt + row + 1);
   const int na = (int)(a1 - a0);
+  np_out = 33;
+  if (na > 32) return false;  // warp-uniform: the grouped path takes this matrix
   long long b0 = 0;
   int len = 0;
   VT av = VT(0);
@@ -161,14 +163,10 @@ __device__ __forceinline__ bool small_warp_row(const int64_t* __restrict__ a_rpt
     len = (int)(__ldg(b_rpt + kk + 1) - b0);
   }
   long long np = len;
-  for (long long j = a0 + 32 + lane; j < a1; j += 32) {  // rows longer than 32: n_prod only
-    const int k2 = __ldg(a_col + j);
-    np += __ldg(b_rpt + k2 + 1) - __ldg(b_rpt + k2);
-  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) np += __shfl_xor_sync(kFullW, np, o);
   np_out = np;
-  if (na > 32 || np > 32) return false;  // warp-uniform
+  if (np > 32) return false;  // warp-uniform
   int incl = len;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {

@@ -102,6 +102,7 @@ struct spgemm_ctx {
   // thread) leaves 8-16 warps per SM and the shuffle stages serialise
   int wsort = 0;
   bool small = false;    // the last symbolic call took the small-matrix path
+  std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
   // 26.5 ms vs 21.7 ms with the per-group hash / rank-count kernels), bit 2 numeric ESC
   int batch = 2;
@@ -628,8 +629,10 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
 
   ALLOC(h->acc, sizeof(DevAcc));
   DevAcc* dacc = static_cast<DevAcc*>(h->acc.p);
+  const std::vector<long long> small_key = {m, k, n, (long long)a_rpt, (long long)a_col, (long long)b_rpt,
+                                             (long long)b_col};
   const bool small_try = h->small_opt && m > 0 && m <= kSmallRows && h->sym_min_group < 0 && h->num_min_group < 0 &&
-                         h->tiny >= 1 && !h->validate;
+                         h->tiny >= 1 && !h->validate && h->small_miss != small_key;
   if (!small_try) {
     CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));
     CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
@@ -716,6 +719,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       CK(leave(h));
       return SPGEMM_OK;
     }
+    h->small_miss = small_key;  // the same inputs go straight to the grouped path next time
     CK(cudaMemsetAsync(c_rpt, 0, sizeof(int64_t), h->stream));  // general path from scratch
     CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
   }
