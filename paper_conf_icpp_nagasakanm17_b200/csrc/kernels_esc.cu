@@ -17,13 +17,14 @@
 //                distinct (n_prod_i <= ESC_PCT/100 * nnz_i) the table is nearly all fixed cost,
 //                so this kernel orders the products themselves: each row's span [lo_i, hi_i] is
 //                cut into next_pow2(n_prod_i) buckets of 2^s columns; a shared-memory counting
-//                pass places every product in its bucket (histogram, exclusive scan, scatter);
+//                pass places every product in its bucket (histogram, exclusive scan, scatter; a
+//                batch whose largest bucket is crowded splits its buckets by the next bits);
 //                inside a bucket (about one product on average) each product takes the paper's
-//                comparison rank (#smaller keys + #equal keys placed before it); equal keys are
-//                then adjacent, the first of each run is the entry (a head), its run is summed in
-//                the working precision, and a scan of the head flags gives every
-//                entry its final position in C.  Output is compact and sorted and
-//                written with coalesced stores.
+//                comparison rank (#smaller keys); the first product of each column is the entry
+//                (a head) and sums the values of its column (working precision);
+//                a scan of the distinct count per bucket plus the head's rank among the bucket's
+//                distinct columns gives every entry its final position in C.  Output is compact
+//                and sorted and written with coalesced stores.
 #include <climits>
 
 #include "spgemm_internal.cuh"
@@ -72,7 +73,6 @@ struct EscRows {
   int bbase[R + 1];    // first bucket (numeric) / first table slot / 4 (symbolic)
   int obase[R + 1];    // first output entry (numeric)
   int nr;              // rows in this batch
-  int maxpos;          // (diagnostic) largest bucket
 };
 
 template <int R, bool NUM>
