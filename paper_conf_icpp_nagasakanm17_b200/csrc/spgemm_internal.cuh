@@ -355,22 +355,33 @@ __device__ __forceinline__ void for_each_product_flat(const int64_t* __restrict_
       if (gl >= d) incl += y;
     }
     const int total = __shfl_sync(gm, incl, G - 1, G);
-    for (int p0 = 0; p0 < total; p0 += G) {
-      const int p = p0 + gl;
-      int e = 0;
+    // kFlatU products per lane per round: all their gathers are issued before the first table
+    // update (the B rows of graph shapes are short and scattered: each gather is an L2/HBM trip)
+    constexpr int kFlatU = 4;
+    for (int p0 = 0; p0 < total; p0 += G * kFlatU) {
+      int keys[kFlatU];
+      VT vals[kFlatU];
 #pragma unroll
-      for (int st = G / 2; st > 0; st >>= 1)
-        if (__shfl_sync(gm, incl, e + st - 1, G) <= p) e += st;
-      const int ie = __shfl_sync(gm, incl, e, G);
-      const int le = __shfl_sync(gm, len, e, G);
-      const long long be = __shfl_sync(gm, b0, e, G);
-      const VT ae = NUM ? __shfl_sync(gm, av, e, G) : VT(0);
-      if (p < total) {
-        const long long q = be + (p - (ie - le));
-        const int key = __ldg(b_col + q);
-        const VT v = NUM ? __ldg(b_val + q) : VT(0);
-        if (!(CHECK_STOP && stop())) f(key, ae * v);
+      for (int u = 0; u < kFlatU; ++u) {
+        const int p = p0 + u * G + gl;
+        int e = 0;
+#pragma unroll
+        for (int st = G / 2; st > 0; st >>= 1)
+          if (__shfl_sync(gm, incl, e + st - 1, G) <= p) e += st;
+        const int ie = __shfl_sync(gm, incl, e, G);
+        const int le = __shfl_sync(gm, len, e, G);
+        const long long be = __shfl_sync(gm, b0, e, G);
+        const VT ae = NUM ? __shfl_sync(gm, av, e, G) : VT(0);
+        keys[u] = -1;
+        if (p < total) {
+          const long long q = be + (p - (ie - le));
+          keys[u] = __ldg(b_col + q);
+          if (NUM) vals[u] = ae * __ldg(b_val + q);
+        }
       }
+#pragma unroll
+      for (int u = 0; u < kFlatU; ++u)
+        if (keys[u] >= 0 && !(CHECK_STOP && stop())) f(keys[u], NUM ? vals[u] : VT(0));
     }
     if constexpr (CHECK_STOP) {
       if (__any_sync(gm, stop())) return;
