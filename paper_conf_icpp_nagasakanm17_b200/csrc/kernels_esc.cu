@@ -275,7 +275,7 @@ template <typename VT>
 __device__ __forceinline__ int swv(int j) { return sizeof(VT) == 8 ? j + (j >> 4) : j + (j >> 5); }
 
 #ifndef SPG_ESC_SKEW
-#define SPG_ESC_SKEW 16
+#define SPG_ESC_SKEW 32
 #endif
 constexpr int kEscSkew = SPG_ESC_SKEW;  // a batch whose largest bucket holds more products is refined
 // BM: coarse buckets per row = BM * next_pow2(n_prod_i) (2, or 1 where shared memory is short);
@@ -622,8 +622,13 @@ constexpr int kEscSmemMax = kSmemLimit - 1024;
 // one coarse bucket per product bound (2 measured slower on R-MAT s22: 55 -> 68 ms, the larger
 // counter scans and clears cost more than the shorter in-bucket ranks save); the refinement where
 // it fits
+#ifndef SPG_ESC_BM
+#define SPG_ESC_BM 1
+#endif
 template <typename VT, int G>
-constexpr int num_esc_bm() { return 1; }
+constexpr int num_esc_bm() {
+  return SPG_ESC_BM > 1 && num_esc_smem_v<VT, G, SPG_ESC_BM, true>() <= kEscSmemMax ? SPG_ESC_BM : 1;
+}
 template <typename VT, int G>
 constexpr bool num_esc_rf() { return num_esc_smem_v<VT, G, num_esc_bm<VT, G>(), true>() <= kEscSmemMax; }
 template <typename VT, int G>
