@@ -278,23 +278,19 @@ __device__ __forceinline__ int swv(int j) { return sizeof(VT) == 8 ? j + (j >> 4
 #define SPG_ESC_SKEW 32
 #endif
 constexpr int kEscSkew = SPG_ESC_SKEW;  // a batch whose largest bucket holds more products is refined
-// BM: coarse buckets per row = BM * next_pow2(n_prod_i) (2, or 1 where shared memory is short);
-// REFINE: the skew refinement (its fine counters) fits
-
-template <typename VT, int TPR, int KP, int MC, int R, int BM, bool REFINE>
+// Shared memory of one batch, sized so that 48 warps fit on an SM (fp32: 1536 / TPR CTAs): the
+// fine counters of the refinement live in sk (dead until the scatter), and the bucket table cnt
+// carries, by phase: coarse counters -> starts -> fine base | bits << 24 (refinement) -> starts
+// (low 16 bits) | duplicate count << 16 (rank) -> start | output base << 16 | has-duplicates << 31.
+template <typename VT, int TPR, int KP, int MC, int R>
 struct NumEscSmem {
   static constexpr int CAP = TPR * KP;
-  static constexpr int NB = BM * CAP;  // coarse (and fine) buckets per batch, at most
-  int sk[CAP + CAP / 32 + 1];   // keys: bucket order, then the compacted output
+  static constexpr int NB = CAP;  // coarse (and fine) buckets per batch, at most
+  int sk[CAP + CAP / 32 + 2];   // keys: bucket order, then the compacted output; fine counters
   VT sv[CAP + CAP / 16 + 1];    // values, same orders
-  alignas(16) int cnt[NB + NB / 32 + 2];  // coarse bucket counters -> starts (-> fine base | bits << 24)
-  int db[NB + NB / 32 + 2];     // distinct entries per bucket -> output base | (bucket has equal keys) << 30
-  unsigned dupw[NB / 2 + 1];    // 16-bit counters: products with an equal key placed before them
+  alignas(16) int cnt[NB + NB / 32 + 2];  // bucket table (above)
   uint16_t sb[CAP];             // bucket of each slot (bucket order); bit 15: the slot heads its key
-  union {                       // the gather's metadata is dead once the products are in registers
-    EscMeta<VT, TPR * MC, CAP> mt;
-    int fcnt[REFINE ? NB + NB / 32 + 2 : 1];  // fine bucket counters -> starts (skewed batches)
-  } u;
+  EscMeta<VT, TPR * MC, CAP> mt;
   EscRows<R> rt;
   int ws[32];
   int smax;
@@ -322,12 +318,16 @@ __device__ __forceinline__ int esc_scan_counts(int* c, int* ws, int (&vals)[N]) 
   return tot;
 }
 
-template <typename VT, int TPR, int KP, int MC, int R, int BM, bool REFINE>
-__global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(NumArgs a) {
-  constexpr int kEscBm = BM;
-  using S = NumEscSmem<VT, TPR, KP, MC, R, BM, REFINE>;
+#ifndef SPG_ESC_OCC
+#define SPG_ESC_OCC 1536
+#endif
+constexpr int kEscOcc = SPG_ESC_OCC;  // fp32 threads per SM the launch bounds ask for
+
+template <typename VT, int TPR, int KP, int MC, int R>
+__global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void k_num_esc(NumArgs a) {
+  using S = NumEscSmem<VT, TPR, KP, MC, R>;
   constexpr int CAP = S::CAP;
-  static_assert(kEscBm * CAP < 65536, "bucket ids and positions are packed into 16 bits each");
+  static_assert(CAP <= 4096, "bucket starts and output bases are packed into 16 and 15 bits");
   extern __shared__ __align__(16) unsigned char smem_raw[];
   S* sm = reinterpret_cast<S*>(smem_raw);
   const int t = threadIdx.x;
@@ -336,14 +336,13 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     int4* c4 = reinterpret_cast<int4*>(sm->cnt);
     for (int i = t; i < (S::NB + S::NB / 32 + 2) / 4; i += TPR) c4[i] = make_int4(0, 0, 0, 0);
     for (int i = ((S::NB + S::NB / 32 + 2) / 4) * 4 + t; i < S::NB + S::NB / 32 + 2; i += TPR) sm->cnt[i] = 0;
-    for (int i = t; i < S::NB / 2 + 1; i += TPR) sm->dupw[i] = 0u;
   }
   if (t == 0) sm->smax = 0;
   __syncthreads();
   const int nr = sm->rt.nr;
   int key[KP], rix[KP];
   VT val[KP];
-  esc_gather<VT, true, TPR, KP, MC, R, CAP>(&sm->rt, &sm->u.mt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
+  esc_gather<VT, true, TPR, KP, MC, R, CAP>(&sm->rt, &sm->mt, a.a_col, static_cast<const VT*>(a.a_val), a.b_rpt,
                                             a.b_col, static_cast<const VT*>(a.b_val), sm->ws, key, val, rix);
   // coarse buckets: bkt = bbase_r + ((key - lo_r) >> sh_r), next_pow2(n_prod_i) per row; pos =
   // arrival order in the bucket
@@ -355,9 +354,9 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     if (key[u] >= 0) {
       const int r = rix[u];
       const unsigned d = (unsigned)(key[u] - sm->rt.lo[r]) >> sm->rt.sh[r];
-      const int nbr = kEscBm * (sm->rt.bbase[r + 1] - sm->rt.bbase[r]);
+      const int nbr = sm->rt.bbase[r + 1] - sm->rt.bbase[r];
       if (d < (unsigned)nbr) {
-        const int bkt = kEscBm * sm->rt.bbase[r] + (int)d;
+        const int bkt = sm->rt.bbase[r] + (int)d;
         const int pos = atomicAdd(&sm->cnt[sw4(bkt)], 1);
         bp[u] = ((unsigned)bkt << 16) | (unsigned)pos;
       } else {
@@ -367,9 +366,9 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
   }
   if (bad) atomicOr(a.err_flags, 2);
   __syncthreads();
-  const int NBt = kEscBm * sm->rt.bbase[nr];
+  const int NBt = sm->rt.bbase[nr];
   const int Pt = sm->rt.pbase[nr];
-  constexpr int KB = kEscBm * KP;  // counters per thread
+  constexpr int KB = KP;  // counters per thread
   {
     int mx = 0;
 #pragma unroll
@@ -380,11 +379,10 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     esc_scan_counts<TPR, KB>(sm->cnt, sm->ws, c);  // (its barriers publish smax)
   }
   __syncthreads();
-  const int* bst = sm->cnt;  // bucket starts used below (coarse, or fine after refinement)
-  if (REFINE && sm->smax > kEscSkew) {
-    // CTA-uniform: split each coarse bucket of n >= 2 products into fine buckets of the next bits
-    // (down to single columns).
-    // ep: 4 bits per coarse bucket of this thread (its fine-bucket bits e, 15 = empty)
+  if (sm->smax > kEscSkew) {
+    // CTA-uniform: split each coarse bucket of n >= 2 products into 2^e fine buckets of the next
+    // bits (down to single columns), e = ceil(log2 n) - 1, so that the fine buckets number at
+    // most n_prod <= NB.  ep: 4 bits per coarse bucket of this thread (e, 15 = empty).
     unsigned long long ep = 0;
     int tot_f = 0;
 #pragma unroll
@@ -395,10 +393,8 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
       if (b < NBt && n > 0) {
         e = 0;
         if (n > 1) {
-          const int r = esc_find<R>(sm->rt.bbase, nr, b / kEscBm);
-          // 2^e fine buckets: e = ceil(log2 n) (BM = 2) or one less (BM = 1), so that the sum of
-          // fine buckets stays below BM * n_prod <= NB
-          e = min(32 - __clz(n - 1) - (BM == 1 ? 1 : 0), sm->rt.sh[r]);
+          const int r = esc_find<R>(sm->rt.bbase, nr, b);
+          e = min(31 - __clz(n - 1), sm->rt.sh[r]);
         }
         tot_f += 1 << e;
       }
@@ -406,31 +402,34 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     }
     int F;
     int run = esc_scan<TPR>(tot_f, &F, sm->ws);  // (every thread has read its counts before it)
+    int* fcnt = sm->sk;  // fine counters (sk is dead until the scatter)
 #pragma unroll
     for (int i = 0; i < KB; ++i) {
       const int e = (int)((ep >> (4 * i)) & 15u);
       sm->cnt[sw4(t * KB + i)] = run | ((e & 15) << 24);  // fine base of coarse bucket t*KB+i, bits
       if (e != 15) run += 1 << e;
     }
-    for (int i = t; i < S::NB + S::NB / 32 + 2; i += TPR) sm->u.fcnt[i] = 0;
+    for (int i = t; i < S::NB + S::NB / 32 + 2; i += TPR) fcnt[i] = 0;
     __syncthreads();
 #pragma unroll
     for (int u = 0; u < KP; ++u)
       if (bp[u] != 0xffffffffu) {
-        const int b = (int)(bp[u] >> 16), r = esc_find<R>(sm->rt.bbase, nr, b / kEscBm);  // (rix is dead here)
+        const int b = (int)(bp[u] >> 16), r = esc_find<R>(sm->rt.bbase, nr, b);  // (rix is dead here)
         const int fe = sm->cnt[sw4(b)];
         const int e = fe >> 24;
         const unsigned rel = (unsigned)(key[u] - sm->rt.lo[r]);
         const int fb = (fe & 0xffffff) + (int)((rel >> (sm->rt.sh[r] - e)) & ((1u << e) - 1u));
-        const int pos = atomicAdd(&sm->u.fcnt[sw4(fb)], 1);
+        const int pos = atomicAdd(&fcnt[sw4(fb)], 1);
         bp[u] = ((unsigned)fb << 16) | (unsigned)pos;
       }
     __syncthreads();
     int c2[KB];
-    esc_scan_counts<TPR, KB>(sm->u.fcnt, sm->ws, c2);
+    esc_scan_counts<TPR, KB>(fcnt, sm->ws, c2);
     __syncthreads();
-    bst = sm->u.fcnt;
+    for (int i = t; i < S::NB + S::NB / 32 + 2; i += TPR) sm->cnt[i] = fcnt[i];
+    __syncthreads();
   }
+  int* const bst = sm->cnt;  // bucket starts (coarse, or fine after refinement)
   // scatter into bucket order (sb: the bucket of every slot)
 #pragma unroll
   for (int u = 0; u < KP; ++u)
@@ -446,7 +445,7 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
   // buckets together: uniform trip counts, broadcast reads): lt = #smaller keys (PAPER.md:173's
   // comparison rank), the slot heads its key when no equal key sits before it; a head sums the
   // values of all equal keys (accumulation in the working precision); a non-head
-  // is counted as a duplicate of its bucket.
+  // is counted as a duplicate of its bucket (high half of its bucket-table word).
   int lt[KP];
 #pragma unroll
   for (int i = 0; i < KP; ++i) {
@@ -454,7 +453,7 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     lt[i] = -1;
     if (j < Pt) {
       const int b = sm->sb[j];
-      const int j0 = bst[sw4(b)], j1 = bst[sw4(b + 1)];
+      const int j0 = bst[sw4(b)] & 0xffff, j1 = bst[sw4(b + 1)] & 0xffff;
       const int k = sm->sk[sw4(j)];
       VT sum = VT(0);
       int l = 0, eqb = 0;
@@ -473,7 +472,7 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
         val[i] = sum;
         sm->sb[j] = (uint16_t)(b | 0x8000);
       } else {
-        atomicAdd(&sm->dupw[b >> 1], 1u << (16 * (b & 1)));
+        atomicAdd(&bst[sw4(b)], 1 << 16);
       }
     }
   }
@@ -481,20 +480,24 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
   // distinct entries per bucket -> exclusive scan (blocked, KB buckets per thread) -> output base
   int H;
   {
-    int d[KB], s = 0;
+    int s = 0;
+    unsigned w0 = (unsigned)bst[sw4(t * KB)];
+#pragma unroll
+    for (int i = 0; i < KB; ++i) {
+      const unsigned w1 = (unsigned)bst[sw4(t * KB + i + 1)];
+      s += t * KB + i < NBt ? (int)(w1 & 0xffffu) - (int)(w0 & 0xffffu) - (int)(w0 >> 16) : 0;
+      w0 = w1;
+    }
+    int run = esc_scan<TPR>(s, &H, sm->ws);  // (every thread has read its words before it)
+    // (a thread rewrites only its own words, after reading them; the low halves stay)
+    w0 = (unsigned)bst[sw4(t * KB)];
 #pragma unroll
     for (int i = 0; i < KB; ++i) {
       const int b = t * KB + i;
-      const int dup = (int)((sm->dupw[b >> 1] >> (16 * (b & 1))) & 0xffffu);
-      d[i] = (b < NBt ? bst[sw4(b + 1)] - bst[sw4(b)] : 0) - dup;
-      s += d[i];
-      d[i] |= dup ? (1 << 30) : 0;
-    }
-    int run = esc_scan<TPR>(s, &H, sm->ws);
-#pragma unroll
-    for (int i = 0; i < KB; ++i) {
-      sm->db[sw4(t * KB + i)] = run | (d[i] & (1 << 30));
-      run += d[i] & ~(1 << 30);
+      const unsigned w1 = (unsigned)bst[sw4(b + 1)], dup = w0 >> 16;
+      bst[sw4(b)] = (int)((w0 & 0xffffu) | ((unsigned)run << 16) | (dup ? 0x80000000u : 0u));
+      run += b < NBt ? (int)(w1 & 0xffffu) - (int)(w0 & 0xffffu) - (int)dup : 0;
+      w0 = w1;
     }
   }
   const int Ot = sm->rt.obase[nr];
@@ -508,15 +511,15 @@ __global__ __launch_bounds__(TPR, (KP >= 8 ? 1024 : 1536) / TPR) void k_num_esc(
     if (lt[i] >= 0) {
       const int j = i * TPR + t;
       const int b = sm->sb[j] & 0x7fff;
-      const int dbb = sm->db[sw4(b)];
+      const unsigned dbb = (unsigned)bst[sw4(b)];
       int dl = lt[i];
-      if (dbb & (1 << 30)) {  // bucket with equal keys: count the smaller heads only
-        const int j0 = bst[sw4(b)], j1 = bst[sw4(b + 1)];
+      if (dbb >> 31) {  // bucket with equal keys: count the smaller heads only
+        const int j0 = (int)(dbb & 0xffffu), j1 = bst[sw4(b + 1)] & 0xffff;
         dl = 0;
 #pragma unroll 1
         for (int q = j0; q < j1; ++q) dl += (sm->sk[sw4(q)] < key[i]) & (sm->sb[q] >> 15);
       }
-      lt[i] = (dbb & ~(1 << 30)) + dl;
+      lt[i] = (int)((dbb >> 16) & 0x7fffu) + dl;
     }
   }
   __syncthreads();
@@ -567,15 +570,18 @@ constexpr int kEscSmallTpr = SPG_ESC_SMALL_TPR;
 #ifndef SPG_ESC_KP
 #define SPG_ESC_KP 8
 #endif
+#ifndef SPG_ESC_MC
+#define SPG_ESC_MC 1
+#endif
 constexpr int kEscKp = SPG_ESC_KP;  // products per thread (fp32); CAP = TPR * KP >= the group bound
 constexpr EscCfg kEscNum32[] = {{0, 0, 0},
                                 {0, 0, 0},
-                                {kEscSmallTpr, kEscKp, 2},
-                                {kEscSmallTpr, kEscKp, 2},
-                                {kEscSmallTpr, kEscKp, 2},
-                                {kEscSmallTpr * 8 / kEscKp >= 128 ? kEscSmallTpr * 8 / kEscKp : 128, kEscKp, 2},
-                                {256 * 8 / kEscKp, kEscKp, 2},
-                                {512 * 8 / kEscKp, kEscKp, 2},
+                                {kEscSmallTpr, kEscKp, SPG_ESC_MC},
+                                {kEscSmallTpr, kEscKp, SPG_ESC_MC},
+                                {kEscSmallTpr, kEscKp, SPG_ESC_MC},
+                                {kEscSmallTpr * 8 / kEscKp >= 128 ? kEscSmallTpr * 8 / kEscKp : 128, kEscKp, SPG_ESC_MC},
+                                {256 * 8 / kEscKp, kEscKp, SPG_ESC_MC},
+                                {512 * 8 / kEscKp, kEscKp, SPG_ESC_MC},
                                 {1024, 8, 2},
                                 {1024, 16, 1}};
 constexpr EscCfg kEscNum64[] = {{0, 0, 0},  {0, 0, 0},  {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
@@ -612,44 +618,28 @@ cudaError_t launch_sym_batch_g(cudaStream_t s, const SymArgs& a) {
   return cudaGetLastError();
 }
 
-template <typename VT, int G, int BM, bool RF>
-constexpr int num_esc_smem_v() {
+template <typename VT, int G>
+constexpr int num_esc_smem_g() {
   constexpr EscCfg c = esc_num_cfg<VT>(G);
   constexpr int R = c.TPR * c.KP / (int)kSymGroups[G].upper;
-  return (int)sizeof(NumEscSmem<VT, c.TPR, c.KP, c.MC, R, BM, RF>);
+  return (int)sizeof(NumEscSmem<VT, c.TPR, c.KP, c.MC, R>);
 }
 constexpr int kEscSmemMax = kSmemLimit - 1024;
-// one coarse bucket per product bound (2 measured slower on R-MAT s22: 55 -> 68 ms, the larger
-// counter scans and clears cost more than the shorter in-bucket ranks save); the refinement where
-// it fits
-#ifndef SPG_ESC_BM
-#define SPG_ESC_BM 1
-#endif
-template <typename VT, int G>
-constexpr int num_esc_bm() {
-  return SPG_ESC_BM > 1 && num_esc_smem_v<VT, G, SPG_ESC_BM, true>() <= kEscSmemMax ? SPG_ESC_BM : 1;
-}
-template <typename VT, int G>
-constexpr bool num_esc_rf() { return num_esc_smem_v<VT, G, num_esc_bm<VT, G>(), true>() <= kEscSmemMax; }
-template <typename VT, int G>
-constexpr int num_esc_smem_g() { return num_esc_smem_v<VT, G, num_esc_bm<VT, G>(), num_esc_rf<VT, G>()>(); }
 
 template <typename VT, int G>
 cudaError_t launch_num_esc_g(cudaStream_t s, const NumArgs& a) {
   constexpr EscCfg c = esc_num_cfg<VT>(G);
   constexpr int R = c.TPR * c.KP / (int)kSymGroups[G].upper;
   static_assert(R >= 1 && R <= 32, "rows per batch");
-  constexpr int BM = num_esc_bm<VT, G>();
-  constexpr bool RF = num_esc_rf<VT, G>();
   constexpr int smem = num_esc_smem_g<VT, G>();
   if constexpr (smem > kEscSmemMax) {
     return cudaErrorInvalidValue;  // the caller does not route these rows here (numeric_esc_supported)
   } else {
     static PerDevice cache;
-    cudaError_t e = esc_prepare(k_num_esc<VT, c.TPR, c.KP, c.MC, R, BM, RF>, smem, cache);
+    cudaError_t e = esc_prepare(k_num_esc<VT, c.TPR, c.KP, c.MC, R>, smem, cache);
     if (e != cudaSuccess) return e;
     const long long grid = (a.nrows + R - 1) / R;
-    k_num_esc<VT, c.TPR, c.KP, c.MC, R, BM, RF><<<(unsigned)grid, c.TPR, smem, s>>>(a);
+    k_num_esc<VT, c.TPR, c.KP, c.MC, R><<<(unsigned)grid, c.TPR, smem, s>>>(a);
     return cudaGetLastError();
   }
 }
