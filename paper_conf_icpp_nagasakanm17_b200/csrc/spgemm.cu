@@ -108,7 +108,7 @@ struct spgemm_ctx {
   int batch = 2;
   long long esc_pct = 200;  // numeric ESC rows: 100 * n_prod_i <= esc_pct * nnz_i
   long long esc_mask = -1;  // symbolic groups whose rows may take the numeric ESC kernels (-1: auto)
-  long long esc_w_pct = 200;  // auto rule: ESC where 100 * (n/1024 + 1) >= esc_w_pct * group bound
+  long long esc_w_pct = 100;  // auto rule: ESC where 100 * (n/1024 + 1) >= esc_w_pct * group bound
   bool phase_streams = true;  // the current phase forks per-group streams (phase_concurrent)
   // CTA-per-row numeric hash groups: two-level bitmap rank (else bucket sort); 1 = only where the
   // level-1 width W <= the group's nnz bound (R-MAT s22, W = 4097: bucket 4.1 ms vs bitmap 21.9 ms
@@ -379,12 +379,12 @@ bool flat_of(spgemm_handle_t h) {
 // Symbolic groups whose weakly compressing rows take the numeric ESC kernels (kernels_esc.cu)
 // instead of the rank-indexed CTA-per-row kernels, whose level-1 bitmap costs W = n/1024 + 1 words
 // per row whatever the row's size: ESC where 100 * W >= esc_w_pct * B (B = the group's n_prod
-// bound).  Measured per group (scripts/esc_groups.py, serial, fp32): R-MAT s22 (W = 4097) ESC
-// saves 1.7 / 1.3 / 3.4 / 5.8 / 2.0 ms on groups 2-6 (W/B = 32 .. 2) and loses 1.8 / 1.9 ms on
-// groups 7-8 (W/B = 1, 0.5); R-MAT s20 (W = 1025) saves 0.4 / 0.1 ms on groups 2-3 (W/B = 8, 4),
-// loses 0.2 ms on group 4 (W/B = 2); webbase, R-MAT s16/s18, Economics, Circuit lose on every
-// group (W <= 1024: their level-1 bitmaps are cheap; webbase's 95 %-local rows also skew the
-// buckets, which costs the ESC kernels a refinement pass).
+// bound).  Measured per group (scripts/esc_groups.py, serial, fp32, ESC at 48 warps per SM):
+// R-MAT s22 (W = 4097) ESC saves 1.9 / 2.0 / 4.8 / 7.8 / 4.2 / 0.8 ms on groups 2-7 (W/B = 32 ..
+// 1) and breaks even on group 8 (W/B = 0.5); R-MAT s20 (W = 1025) saves 0.46 / 0.26 / 0.10 /
+// 0.08 ms on groups 2-5 (W/B = 8 .. 1), loses 0.23 ms on group 6 (W/B = 0.5); webbase, R-MAT
+// s16/s18, Economics, Circuit lose on most groups (W <= 1024: their level-1 bitmaps are cheap;
+// webbase's 95 %-local rows also skew the buckets, which costs the ESC kernels a refinement pass).
 unsigned esc_auto_mask(spgemm_handle_t h) {
   const long long W = h->n / 1024 + 1;
   unsigned m = 0;

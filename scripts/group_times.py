@@ -31,3 +31,12 @@ with P.Handle() as h:
           f"num {st['numeric_ms']:.2f}")
     print("   sym " + " ".join(f"g{g}:{st['sym_group_ms'][g]:.2f}" for g in range(24) if st["sym_group_ms"][g] > 0))
     print("   num " + " ".join(f"g{g}:{st['num_group_ms'][g]:.2f}" for g in range(24) if st["num_group_ms"][g] > 0))
+    if os.environ.get("GT_DETAIL"):
+        for ph in ("sym", "num"):
+            for g in range(24):
+                ms = st[f"{ph}_group_ms"][g]
+                if ms > 0:
+                    rows, npr = st[f"{ph}_rows"][g], st[f"{ph}_nprod"][g]
+                    nnzc = st["num_nnzc"][g] if ph == "num" else 0
+                    print(f"   {ph} g{g:2d} kind {st[f'{ph}_kernel'][g] if f'{ph}_kernel' in st else '?'} rows {rows:9d} "
+                          f"nprod {npr:12d} nnzc {nnzc:12d} ms {ms:7.3f} Gprod/s {npr / ms / 1e6:7.1f}")
