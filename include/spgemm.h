@@ -197,6 +197,14 @@ typedef enum {
                                        a bitonic-sorted register row; 2 = numeric rows of those groups
                                        with 100 * n_prod_i <= ESC_PCT * nnz_i.  Default 0 (measured
                                        slower than the hash / ESC kernels: ablation) */
+    SPGEMM_OPT_RANK_BIG_SYM = 26,   /* 1 (default): symbolic rows above the last n_prod bound (the
+                                       optimistic group) are counted exactly by one 1024-thread CTA
+                                       per row with the two-level bitmap of RANK_ACC, level 2 in
+                                       chunks of 32768 blocks, when the group has
+                                       at least 4 rows per SM; 2: whatever its size.  Needs
+                                       RANK_ACC and the column spans.  0: the paper's chain — optimistic shared
+                                       table, overflow rows recounted in cluster / global tables
+                                        */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,

@@ -227,11 +227,13 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
     const unsigned w = d >> 10, bit = (d >> 5) & 31;
     return (int)p1[w] + __popc(l1[w] & ((1u << bit) - 1u));
   };
-  auto set_fine = [&](int k) {
+  // level 2 of the blocks with compact index in [c0, c0 + UPPER) (symbolic rows with more
+  // non-empty blocks than UPPER take them in chunks; numeric: c0 = 0 and nb <= UPPER)
+  auto set_fine = [&](int k, int c0) {
     const unsigned d = (unsigned)(k - lo);
-    const int b = blk_of(d);
+    const int b = blk_of(d) - c0;
     const unsigned bit = 1u << (d & 31);
-    if (!(fine[b] & bit)) atomicOr(fine + b, bit);
+    if ((NUM || (unsigned)b < (unsigned)UPPER) && !(fine[b] & bit)) atomicOr(fine + b, bit);
   };
   auto accumulate = [&](int k, VT v) {
     const unsigned d = (unsigned)(k - lo);
@@ -270,27 +272,34 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   __syncthreads();
   // (iii) compact index of the non-empty 32-column blocks
   const int nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
-  const bool ok = nb <= (int)UPPER;  // CTA-uniform; false only for inconsistent input
-  if (ok) clear_words<TPR>(fine, nb);
-  __syncthreads();
-  // (iv) level 2
-  if (ok) {
+  // CTA-uniform; numeric: false only for inconsistent input (the symbolic count bounds nb)
+  const bool ok = !NUM || nb <= (int)UPPER;
+  auto level2 = [&](int c0) {
     if (fast) {
 #pragma unroll
       for (int u = 0; u < KP; ++u)
-        if (key[u] >= 0) set_fine(key[u]);
+        if (key[u] >= 0) set_fine(key[u], c0);
     } else {
-      walk([&](int k, VT) { set_fine(k); });
+      walk([&](int k, VT) { set_fine(k, c0); });
     }
-  }
+  };
+  if (ok) clear_words<TPR>(fine, min(nb, (int)UPPER));
+  __syncthreads();
+  // (iv) level 2
+  if (ok) level2(0);
   __syncthreads();
   if constexpr (!NUM) {
-    // symbolic: nnz_i = number of distinct columns = popcount of level 2
-    const int n = ok ? prefix_popc<TPR>(fine, nb, nullptr, ws32[0]) : 0;
-    if (t == 0) {
-      a.c_cnt[row] = n;
-      if (!ok) atomicOr(a.err_flags, 1);
+    // symbolic: nnz_i = number of distinct columns = popcount of level 2, chunk by chunk
+    int n = prefix_popc<TPR>(fine, min(nb, (int)UPPER), nullptr, ws32[0]);
+    for (int c0 = (int)UPPER; c0 < nb; c0 += (int)UPPER) {  // CTA-uniform
+      __syncthreads();
+      clear_words<TPR>(fine, min(nb - c0, (int)UPPER));
+      __syncthreads();
+      level2(c0);
+      __syncthreads();
+      n += prefix_popc<TPR>(fine, min(nb - c0, (int)UPPER), nullptr, ws32[(c0 / (int)UPPER) & 1]);
     }
+    if (t == 0) a.c_cnt[row] = n;
   } else {
     const long long c0 = a.c_rpt[row];
     const int cn = (int)(a.c_rpt[row + 1] - c0);
@@ -382,6 +391,20 @@ cudaError_t launch_rankcnt_k(cudaStream_t s, const SymArgs& a) {
   cudaError_t e = prepare(k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
   k_sym_rankcnt<c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+// Rows above the last symbolic bound (n_prod_i > 16384, the optimistic group): exact count in one
+// CTA of 1024 threads whatever the row — level 2 in chunks of kRankBigSymUpper blocks, products
+// re-walked per pass — instead of the optimistic table and its cluster / global retries.
+constexpr long long kRankBigSymUpper = 32768;
+using RankBigSymL = RankLayout<int, false, 1024, kRankBigSymUpper, 2, 16>;
+cudaError_t launch_rankcnt_big(cudaStream_t s, const SymArgs& a) {
+  const int smem = RankBigSymL::bytes(a.l1_words);
+  static PerDevice configured;
+  cudaError_t e = prepare(k_sym_rankcnt<1024, kRankBigSymUpper, 16, 2>, smem, configured);
+  if (e != cudaSuccess) return e;
+  k_sym_rankcnt<1024, kRankBigSymUpper, 16, 2><<<(unsigned)a.nrows, 1024, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -533,6 +556,7 @@ int rankacc_smem_bytes(int group, bool fp64, int l1_words) {
 
 int rankcnt_smem_bytes(int group, int l1_words) {
   switch (group) {
+    case kSymOptimistic: return kStaticRankBytes + RankBigSymL::bytes(l1_words);
 #define SPG_G(I)                                                                                  \
   case I:                                                                                         \
     return kStaticRankBytes + RankLayout<int, false, kRankSym[I].TPR, kSymGroups[I].upper,        \
@@ -560,6 +584,7 @@ cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, 
 cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a) {
   if (a.nrows <= 0) return cudaSuccess;
   switch (group) {
+    case kSymOptimistic: return launch_rankcnt_big(s, a);
 #define SPG_G(I) \
   case I: return launch_rankcnt_k<I>(s, a);
     SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)

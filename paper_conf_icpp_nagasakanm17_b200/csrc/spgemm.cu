@@ -101,6 +101,9 @@ struct spgemm_ctx {
   // Economics, Circuit; scripts/ab.py): the unrolled networks' register footprint (up to 240 per
   // thread) leaves 8-16 warps per SM and the shuffle stages serialise
   int wsort = 0;
+  // symbolic optimistic-group rows counted exactly by the chunked rank-count kernel (R-MAT s22:
+  // 1811 rows with n_prod_i > 16384)
+  int rank_big_sym = 1;
   bool small = false;    // the last symbolic call took the small-matrix path
   std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
@@ -592,6 +595,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->esc_pct = v; break;
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_BIG_SYM:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_SYM must be 0, 1 or 2");
+      h->rank_big_sym = (int)v; break;
     case SPGEMM_OPT_WSORT:
       if (v < 0 || v > 3) return fail(h, SPGEMM_ERR_INVALID_ARG, "WSORT must be 0..3");
       h->wsort = (int)v; break;
@@ -746,7 +752,14 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
 
   const Offsets off1 = offsets_of(h->snap1.sym_rows, kNumSymGroups);
   // (3) symbolic hash counting per group
-  const long long n_opt = (long long)h->snap1.sym_rows[kSymOptimistic];
+  // optimistic-group rows counted exactly by the chunked rank-count kernel need no overflow lists
+  // or global slabs (rank_cnt_on(kSymOptimistic) below).  Only with >= 4 rows per SM: one CTA per
+  // row walks its products twice, so a handful of rows leaves the GPU idle behind the largest
+  // (measured: R-MAT s22, 1811 rows, 1.95 -> 0.65 ms; s20, 211 rows, 0.04 -> 0.10 ms)
+  const bool opt_exact = h->rank_acc && h->rank_big_sym && h->rlohi.p != nullptr && h->sym_min_group < 0 &&
+                         (h->rank_big_sym == 2 || (long long)h->snap1.sym_rows[kSymOptimistic] >= 4LL * h->num_sms) &&
+                         rankcnt_smem_bytes(kSymOptimistic, (int)((n + 1023) / 1024 + 1)) <= kSmemLimit;
+  const long long n_opt = opt_exact ? 0 : (long long)h->snap1.sym_rows[kSymOptimistic];
   const long long n_glob = (long long)h->snap1.sym_rows[kSymGlobal];
   if (n_opt > 0) {
     ALLOC(h->overflow, sizeof(int32_t) * n_opt);
@@ -789,6 +802,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   auto wsort_sym_on = [&](int g) { return (h->wsort & 1) && h->sym_min_group < 0 && g >= 2 && g <= wsort_max_group(); };
   // rank-count kernels for the CTA-per-row groups (kernels_rankacc.cu; needs the column spans)
   auto rank_cnt_on = [&](int g) {
+    if (g == kSymOptimistic) return opt_exact;  // level 1 costs W words against > 16384 products
     return h->rank_acc && h->rlohi.p != nullptr && h->sym_min_group < 0 && g >= 5 && g <= 9 &&
            rankcnt_smem_bytes(g, sa.l1_words) <= kSmemLimit &&
            (h->rank_l1_pct_sym == 0 || 100LL * sa.l1_words <= h->rank_l1_pct_sym * kSymGroups[g].upper);
@@ -823,7 +837,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
                                  h->snap1.range_rmax, h->snap1.b_unsorted, (long long)h->range_num, range_bw,
                                  (long long)h->rank_acc, (long long)h->tiny, h->rank_l1_pct_sym,
                                  (long long)h->sym_min_group, (long long)h->batch, h->esc_pct, h->esc_mask,
-                                 (long long)h->small_opt, (long long)h->wsort};
+                                 (long long)h->small_opt, (long long)h->wsort, (long long)h->rank_big_sym};
   for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap1.sym_rows[g]);
   const std::vector<long long> ptrs = {(long long)a_rpt, (long long)a_col, (long long)b_rpt, (long long)b_col,
                                        (long long)c_rpt, (long long)h->perm1.p, (long long)h->acc.p,
@@ -859,7 +873,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       h->gkind[0][g] = tiny_g ? SPGEMM_KERNEL_TINY : wsort_sym_on(g) ? SPGEMM_KERNEL_WSORT : batch_sym_on(g) ? SPGEMM_KERNEL_BATCH
                      : rank_cnt_on(g) ? SPGEMM_KERNEL_RANK : SPGEMM_KERNEL_HASH;
       ++launches;
-      if (g == kSymOptimistic) {  // PAPER.md:155 "After this first phase ... global memory"
+      if (g == kSymOptimistic && !opt_exact) {  // PAPER.md:155 "After this first phase ... global memory"
         SymArgs gb = sa;
         gb.rows = perm1 + off1.off[kSymGlobal];
         gb.nrows = n_glob;

@@ -665,6 +665,26 @@ def test_rank_acc_big_rows(spg, dtype):
     check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
 
 
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_rank_count_big_rows_chunked(spg, dtype):
+    """Symbolic rows above the last n_prod bound (group 10) counted exactly by the rank-count
+    kernel: rows with more than 32768 non-empty 32-column blocks take level 2 in chunks; with
+    RANK_BIG_SYM 0 the same rows go through the paper's optimistic -> cluster -> global chain."""
+    A, B = _big_rows(33)
+    A, B = A.with_values("uniform", 1), B.with_values("uniform", 2)
+    # non-empty 32-column blocks per row of C (the chunking must be exercised)
+    blocks = [np.unique(B.col[np.concatenate([np.arange(B.rpt[k], B.rpt[k + 1])
+                                              for k in A.col[A.rpt[i]:A.rpt[i + 1]]])] >> 5).size
+              for i in range(A.m)]
+    assert max(blocks) > 32768, max(blocks)
+    got = check(spg, A, B, dtype, opts={"rank_big_sym": 2}, what="big rows exact count")
+    st = got[3]
+    assert st["sym_rows"][10] > 0 and st["sym_kernel"][10] == 2, (st["sym_rows"][10], st["sym_kernel"])
+    assert st["sym_overflow_rows"] == 0
+    got = check(spg, A, B, dtype, opts={"rank_big_sym": 0}, what="big rows optimistic chain")
+    assert got[3]["sym_kernel"][10] == 1 and got[3]["sym_overflow_rows"] > 0
+
+
 def test_rank_acc_big_rows_int_exact(spg):
     A, B = _big_rows(32)
     check(spg, A.with_values("int", 3), B.with_values("int", 4), np.float32, exact=True, what="big rows int")
