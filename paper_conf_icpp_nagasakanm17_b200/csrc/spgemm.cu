@@ -33,13 +33,27 @@ struct Buf {
   size_t bytes = 0;
 };
 
-struct GraphCache {
+struct GraphEntry {
   cudaGraphExec_t exec = nullptr;
   std::vector<long long> key;    // full key: topology + every pointer the kernels see
   std::vector<long long> topo;   // topology key: launch structure only (grids, groups, options)
   int launches = 0;              // kernels in the captured segment
   bool timed[16] = {};           // groups with timing events in the segment
   int kind[16] = {};             // spgemm_kernel_t of every group in the segment
+};
+// The active (most recent) entry plus up to kGraphSpare others, most recent first: callers that
+// alternate output buffers (a caching allocator hands back two or three addresses in turn) replay
+// an instantiated graph instead of re-capturing and updating one every call.
+constexpr size_t kGraphSpare = 3;
+struct GraphCache : GraphEntry {
+  std::vector<GraphEntry> others;
+  void destroy() {
+    if (exec) cudaGraphExecDestroy(exec);
+    exec = nullptr;
+    for (GraphEntry& e : others)
+      if (e.exec) cudaGraphExecDestroy(e.exec);
+    others.clear();
+  }
 };
 
 struct DeviceGuard {
@@ -230,10 +244,33 @@ spgemm_status_t run_graph(spgemm_handle_t h, GraphCache& gc, const std::vector<l
   if (!graphs_on(h)) return enqueue();
   std::vector<long long> key = topo;
   key.insert(key.end(), ptrs.begin(), ptrs.end());
+  if (!(gc.exec && gc.key == key)) {  // an older entry of the same call becomes the active one
+    for (size_t i = 0; i < gc.others.size(); ++i)
+      if (gc.others[i].exec && gc.others[i].key == key) {
+        GraphEntry hit = std::move(gc.others[i]);
+        gc.others.erase(gc.others.begin() + (long)i);
+        gc.others.insert(gc.others.begin(), std::move(static_cast<GraphEntry&>(gc)));
+        static_cast<GraphEntry&>(gc) = std::move(hit);
+        break;
+      }
+  }
   if (gc.exec && gc.key == key) {  // identical call: replay
     CK(cudaGraphLaunch(gc.exec, h->stream));
     ++h->stats.graph_replays;
     return SPGEMM_OK;
+  }
+  // a new call: keep the active entry while there is room, else recycle the least recently used
+  // entry (updated in place when its topology matches, else re-instantiated)
+  if (gc.exec) {
+    gc.others.insert(gc.others.begin(), std::move(static_cast<GraphEntry&>(gc)));
+    static_cast<GraphEntry&>(gc) = GraphEntry{};
+    if (gc.others.size() > kGraphSpare) {
+      size_t v = gc.others.size() - 1;  // LRU, or the least recent one with the same topology
+      for (size_t i = gc.others.size(); i-- > 0;)
+        if (gc.others[i].topo == topo) { v = i; break; }
+      static_cast<GraphEntry&>(gc) = std::move(gc.others[v]);
+      gc.others.erase(gc.others.begin() + (long)v);
+    }
   }
   cudaGraph_t g = nullptr;
   CK(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
@@ -508,9 +545,9 @@ spgemm_status_t spgemm_destroy(spgemm_handle_t h) {
       free_all(h);
       cudaStreamSynchronize(h->stream);
     }
-    if (h->gsym.exec) cudaGraphExecDestroy(h->gsym.exec);
-    if (h->gnum.exec) cudaGraphExecDestroy(h->gnum.exec);
-    if (h->gsmall.exec) cudaGraphExecDestroy(h->gsmall.exec);
+    h->gsym.destroy();
+    h->gnum.destroy();
+    h->gsmall.destroy();
     for (int i = 0; i < kNumStreams; ++i) {
       if (h->gs[i]) cudaStreamDestroy(h->gs[i]);
       if (h->join_ev[i]) cudaEventDestroy(h->join_ev[i]);

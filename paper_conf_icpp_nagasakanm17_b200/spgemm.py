@@ -127,6 +127,14 @@ class Handle:
                                          off.ctypes.data_as(ctypes.c_void_p)), self._h, "spgemm_get_grouping")
         return nprod, perm, off
 
+    def _empty(self, n: int, dtype) -> torch.Tensor:
+        """Device buffer from torch's caching allocator, associated with the handle's stream
+        (no stream switch when that is already the current stream)."""
+        if torch.cuda.current_stream(self.device) == self.stream:
+            return torch.empty(n, dtype=dtype, device=self.device)
+        with torch.cuda.stream(self.stream):
+            return torch.empty(n, dtype=dtype, device=self.device)
+
     # ----------------------------------------------------------------- the two phases
     def symbolic(self, A: CsrMatrix, B: CsrMatrix, c_rpt: Optional[torch.Tensor] = None):
         """Phase 1 (PAPER.md:80 steps (1)-(4)): returns (c_rpt, nnz(C), sum n_prod)."""
@@ -135,8 +143,7 @@ class Handle:
         if A.n != B.m:
             raise ValueError(f"shape mismatch: A is {A.m}x{A.n}, B is {B.m}x{B.n}")
         if c_rpt is None:
-            with torch.cuda.stream(self.stream):
-                c_rpt = torch.empty(A.m + 1, dtype=torch.int64, device=self.device)
+            c_rpt = self._empty(A.m + 1, torch.int64)
         nnz = ctypes.c_int64()
         nprod = ctypes.c_int64()
         st = load().spgemm_symbolic(self._h, A.m, B.m, B.n, _ptr(A.rpt), _ptr(A.col), _ptr(B.rpt), _ptr(B.col),
@@ -161,10 +168,8 @@ class Handle:
     def multiply(self, A: CsrMatrix, B: CsrMatrix) -> CsrMatrix:
         """C = A * B with C allocated to its exact nnz."""
         c_rpt, nnz, _ = self.symbolic(A, B)
-        dtype = A.val.dtype
-        with torch.cuda.stream(self.stream):
-            c_col = torch.empty(nnz, dtype=torch.int32, device=self.device)
-            c_val = torch.empty(nnz, dtype=dtype, device=self.device)
+        c_col = self._empty(nnz, torch.int32)
+        c_val = self._empty(nnz, A.val.dtype)
         self.numeric(A.val, B.val, c_col, c_val)
         return CsrMatrix(A.m, B.n, c_rpt, c_col, c_val)
 

@@ -13,9 +13,8 @@ for _ in range(300):
     t0 = time.perf_counter()
     c_rpt, nnz, _ = h.symbolic(dA, dA)
     t1 = time.perf_counter()
-    with torch.cuda.stream(h.stream):
-        c_col = torch.empty(nnz, dtype=torch.int32, device="cuda")
-        c_val = torch.empty(nnz, dtype=torch.float64, device="cuda")
+    c_col = h._empty(nnz, torch.int32)
+    c_val = h._empty(nnz, torch.float64)
     t2 = time.perf_counter()
     h.numeric(dA.val, dA.val, c_col, c_val)
     t3 = time.perf_counter()

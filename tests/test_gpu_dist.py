@@ -88,3 +88,46 @@ def test_bench_sharded_two_ranks_gloo(tmp_path):
     sp = line["multi_gpu"]["splits"]
     assert sp[0] == 0 and sp[-1] == A.m and len(sp) == 3
     assert line["e2e"]["value"] > 0 and line["gpu_launches"] > 0
+
+
+def _nccl_worker(rank, world, port, out_dir):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", 0))
+    try:
+        import synth
+        import paper_conf_icpp_nagasakanm17_b200 as P
+        from paper_conf_icpp_nagasakanm17_b200.dist import (broadcast_csr, cuda_local_multiply, cuda_partition,
+                                                            distributed_spgemm)
+        A = P.CsrMatrix.from_host(synth.config("webbase", "int"), "cuda:0", torch.float32)
+        B = broadcast_csr(A, 0, "cuda:0", torch.float32)  # NCCL chunked broadcast (sizes, rpt, col, val)
+        with P.Handle(0) as h:
+            res, grpt = distributed_spgemm(A, B, device="cuda:0", dtype=torch.float32, square=False,
+                                           partition=cuda_partition(h), local_multiply=cuda_local_multiply(h),
+                                           gather_rpt=True)
+            torch.cuda.synchronize()
+            rpt, col, val = res.C.numpy()
+        np.savez(os.path.join(out_dir, "nccl.npz"), col=col, val=val, grpt=grpt.cpu().numpy(),
+                 nprod=res.nprod, total=res.nnz_total, b_equal=int(torch.equal(B.col, A.col)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_backend_world_one(tmp_path):
+    """The product's collective calls (chunked broadcast of B, all_gather of the shard counts and
+    rpt blocks) on the NCCL backend — one rank on the box's one GPU (ranks that wait on each other
+    must not share a GPU); results equal the oracle bit-exactly (int values)."""
+    import oracle
+    import synth
+    if not torch.cuda.is_available():
+        pytest.fail("needs a GPU")
+    mp.spawn(_nccl_worker, args=(1, _port(), str(tmp_path)), nprocs=1, join=True)
+    H = synth.config("webbase", "int").astype(np.float32)
+    r_rpt, r_col, r_val, _ = oracle.spgemm(H, H, np.float32)
+    got = np.load(os.path.join(tmp_path, "nccl.npz"))
+    assert int(got["b_equal"]) == 1
+    assert np.array_equal(got["grpt"], r_rpt)
+    assert np.array_equal(got["col"], r_col) and np.array_equal(got["val"], r_val)
+    assert int(got["total"]) == r_col.size
