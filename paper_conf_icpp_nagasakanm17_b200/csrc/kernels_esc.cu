@@ -274,6 +274,15 @@ __device__ __forceinline__ int sw4(int j) { return j + (j >> 5); }
 template <typename VT>
 __device__ __forceinline__ int swv(int j) { return sizeof(VT) == 8 ? j + (j >> 4) : j + (j >> 5); }
 
+#ifndef SPG_ESC_V3
+#define SPG_ESC_V3 1
+#endif
+// Key / value slots of sk / sv are only ever read striped (lane-consecutive) or at scattered
+// slots, never blocked, so they need no swizzle (the fine counters that alias sk keep sw4).
+__device__ __forceinline__ int kix(int j) { return SPG_ESC_V3 ? j : sw4(j); }
+template <typename VT>
+__device__ __forceinline__ int vix(int j) { return SPG_ESC_V3 ? j : swv<VT>(j); }
+
 #ifndef SPG_ESC_SKEW
 #define SPG_ESC_SKEW 32
 #endif
@@ -436,8 +445,8 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
     if (bp[u] != 0xffffffffu) {
       const int b = (int)(bp[u] >> 16);
       const int slot = bst[sw4(b)] + (int)(bp[u] & 0xffffu);
-      sm->sk[sw4(slot)] = key[u];
-      sm->sv[swv<VT>(slot)] = val[u];
+      sm->sk[kix(slot)] = key[u];
+      sm->sv[vix<VT>(slot)] = val[u];
       sm->sb[slot] = (uint16_t)b;
     }
   __syncthreads();
@@ -454,9 +463,37 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
     if (j < Pt) {
       const int b = sm->sb[j];
       const int j0 = bst[sw4(b)] & 0xffff, j1 = bst[sw4(b + 1)] & 0xffff;
-      const int k = sm->sk[sw4(j)];
+      const int k = sm->sk[kix(j)];
       VT sum = VT(0);
       int l = 0, eqb = 0;
+#if SPG_ESC_V3
+      // branch-free pass (two slots per step): #smaller keys and #equal keys (itself included);
+      // the values of equal keys are summed in a second pass only where a key repeats (rare for
+      // weakly compressing rows)
+      int ne = 0;
+      int q = j0;
+#pragma unroll 1
+      for (; q + 1 < j1; q += 2) {
+        const int k2 = sm->sk[q], k3 = sm->sk[q + 1];
+        l += (k2 < k) + (k3 < k);
+        ne += (k2 == k) + (k3 == k);
+      }
+      if (q < j1) {
+        const int k2 = sm->sk[q];
+        l += k2 < k;
+        ne += k2 == k;
+      }
+      if (ne == 1) {
+        sum = sm->sv[j];
+      } else {
+#pragma unroll 1
+        for (int q2 = j0; q2 < j1; ++q2)
+          if (sm->sk[q2] == k) {
+            eqb += q2 < j;
+            sum += sm->sv[q2];
+          }
+      }
+#else
 #pragma unroll 1
       for (int q = j0; q < j1; ++q) {
         const int k2 = sm->sk[sw4(q)];
@@ -466,6 +503,7 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
           sum += sm->sv[swv<VT>(q)];
         }
       }
+#endif
       if (eqb == 0) {
         lt[i] = l;
         key[i] = k;
@@ -517,7 +555,7 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
         const int j0 = (int)(dbb & 0xffffu), j1 = bst[sw4(b + 1)] & 0xffff;
         dl = 0;
 #pragma unroll 1
-        for (int q = j0; q < j1; ++q) dl += (sm->sk[sw4(q)] < key[i]) & (sm->sb[q] >> 15);
+        for (int q = j0; q < j1; ++q) dl += (sm->sk[kix(q)] < key[i]) & (sm->sb[q] >> 15);
       }
       lt[i] = (int)((dbb >> 16) & 0x7fffu) + dl;
     }
@@ -527,8 +565,8 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
 #pragma unroll
     for (int i = 0; i < KP; ++i)
       if (lt[i] >= 0) {
-        sm->sk[sw4(lt[i])] = key[i];
-        sm->sv[swv<VT>(lt[i])] = val[i];
+        sm->sk[kix(lt[i])] = key[i];
+        sm->sv[vix<VT>(lt[i])] = val[i];
       }
   }
   __syncthreads();
@@ -540,16 +578,16 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void
     int32_t* __restrict__ c1 = cc + sm->rt.c0[0];
     VT* __restrict__ v1 = cv + sm->rt.c0[0];
     for (int o = t; o < Ot; o += TPR) {
-      c1[o] = sm->sk[sw4(o)];
-      v1[o] = sm->sv[swv<VT>(o)];
+      c1[o] = sm->sk[kix(o)];
+      v1[o] = sm->sv[vix<VT>(o)];
     }
   } else {
     int r = t < Ot ? esc_find<R>(sm->rt.obase, nr, t) : 0;
     for (int o = t; o < Ot; o += TPR) {
       while (sm->rt.obase[r + 1] <= o) ++r;
       const long long dst = sm->rt.c0[r] + (o - sm->rt.obase[r]);
-      cc[dst] = sm->sk[sw4(o)];
-      cv[dst] = sm->sv[swv<VT>(o)];
+      cc[dst] = sm->sk[kix(o)];
+      cv[dst] = sm->sv[vix<VT>(o)];
     }
   }
 }
