@@ -205,6 +205,10 @@ typedef enum {
                                        RANK_ACC and the column spans.  0: the paper's chain — optimistic shared
                                        table, overflow rows recounted in cluster / global tables
                                         */
+    SPGEMM_OPT_RANK_BIG_SHARED = 27,/* 1 (default): numeric rows of group 10 (8192 < nnz_i <= 24576)
+                                       on the rank-big kernel keep the level-2 bitmap and its
+                                       prefix in shared memory when they fit beside level 1
+                                       (DESIGN.md §5.8); 0: in the per-CTA global slab */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,

@@ -34,6 +34,7 @@
 // column span (range hash disabled), for the forced-group paths and as the ablation
 // (SPGEMM_OPT_RANK_ACC = 0).
 #include <climits>
+#include <type_traits>
 
 #include "spgemm_internal.cuh"
 
@@ -98,6 +99,30 @@ __device__ __forceinline__ int prefix_popc(const unsigned* words, int W, uint16_
   return total;
 }
 
+// u32 variant (prefix values above 65535; `global`: the words live in a global slab, read via L2)
+template <int TPR>
+__device__ __forceinline__ int prefix_popc32(const unsigned* words, int W, unsigned* pre, int* ws32, bool global) {
+  const int W4 = (W + 3) >> 2;
+  const int per = (W4 + TPR - 1) / TPR;
+  const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
+  const uint4* w4 = reinterpret_cast<const uint4*>(words);
+  auto ld = [&](int v) { return global ? __ldcg(w4 + v) : w4[v]; };
+  int loc = 0;
+  for (int v = v0; v < v1; ++v) loc += popc4(ld(v));
+  int total;
+  int run = cta_scan32<TPR>(loc, &total, ws32);
+  for (int v = v0; v < v1; ++v) {
+    const uint4 x = ld(v);
+    uint4 o;
+    o.x = (unsigned)run; run += __popc(x.x);
+    o.y = (unsigned)run; run += __popc(x.y);
+    o.z = (unsigned)run; run += __popc(x.z);
+    o.w = (unsigned)run; run += __popc(x.w);
+    reinterpret_cast<uint4*>(pre)[v] = o;
+  }
+  return total;
+}
+
 template <int TPR>
 __device__ __forceinline__ void clear_words(unsigned* words, int W) {
   uint4* w4 = reinterpret_cast<uint4*>(words);
@@ -107,7 +132,8 @@ __device__ __forceinline__ void clear_words(unsigned* words, int W) {
 // Shared-memory layout of one row (16-byte aligned pieces); VT = value type (int: symbolic).
 //   vals[UPPER] VT (numeric) | b0[ME] i64 | av[ME] VT (numeric) | incl[ME] i32 |
 //   keys[UPPER] i32 (numeric) | fine[UPPER] u32 | bstart[KP*TPR/32+1] i32 | l1[L1W] u32 |
-//   pre2[UPPER] u16 (numeric) | p1[L1W] u16
+//   pre2[UPPER] u16 (numeric) | p1[L1W] u16 (u32 for the chunked big-row count: more than
+//   65535 non-empty blocks)
 template <typename VT, bool NUM, int TPR, long long UPPER, int MC, int KP>
 struct RankLayout {
   static constexpr int ME = MC * TPR;  // metadata entries
@@ -121,7 +147,8 @@ struct RankLayout {
   static constexpr int kL1 = kBstart + align16((KP * TPR / 32 + 1) * 4);
   static __host__ __device__ constexpr int pre2(int l1w) { return kL1 + align16(l1w * 4); }
   static __host__ __device__ constexpr int p1(int l1w) { return pre2(l1w) + (NUM ? align16((int)UPPER * 2) : 0); }
-  static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1w * 2); }
+  using P1T = std::conditional_t<(!NUM && UPPER > 16384), unsigned, uint16_t>;
+  static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1w * (int)sizeof(P1T)); }
 };
 
 // Per-group launch shape of the rank kernels (independent of the hash groups' Table-I shapes):
@@ -169,7 +196,8 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   int* bstart = reinterpret_cast<int*>(smem_raw + L::kBstart);
   unsigned* l1 = reinterpret_cast<unsigned*>(smem_raw + L::kL1);
   uint16_t* pre2 = reinterpret_cast<uint16_t*>(smem_raw + L::pre2(a.l1_words));
-  uint16_t* p1 = reinterpret_cast<uint16_t*>(smem_raw + L::p1(a.l1_words));
+  using P1T = typename L::P1T;
+  P1T* p1 = reinterpret_cast<P1T*>(smem_raw + L::p1(a.l1_words));
 
   const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val_ptr());
   const VT* __restrict__ bv_g = static_cast<const VT*>(a.b_val_ptr());
@@ -271,7 +299,9 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   }
   __syncthreads();
   // (iii) compact index of the non-empty 32-column blocks
-  const int nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
+  int nb;
+  if constexpr (sizeof(P1T) == 4) nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
+  else nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
   // CTA-uniform; numeric: false only for inconsistent input (the symbolic count bounds nb)
   const bool ok = !NUM || nb <= (int)UPPER;
   auto level2 = [&](int c0) {
@@ -427,33 +457,14 @@ cudaError_t launch_rankacc_v(cudaStream_t s, int group, const NumArgs& a) {
 // (red.global.add, working precision) after the row is zeroed, keys stored there too.  Products
 // are walked three times (level 1, level 2, accumulate) with the chunked block loop; the second
 // and third walks re-gather B rows that the first one brought into L2.
-template <int TPR>
-__device__ __forceinline__ int prefix_popc32(const unsigned* words, int W, unsigned* pre, int* ws32, bool global) {
-  const int W4 = (W + 3) >> 2;
-  const int per = (W4 + TPR - 1) / TPR;
-  const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
-  const uint4* w4 = reinterpret_cast<const uint4*>(words);
-  auto ld = [&](int v) { return global ? __ldcg(w4 + v) : w4[v]; };
-  int loc = 0;
-  for (int v = v0; v < v1; ++v) loc += popc4(ld(v));
-  int total;
-  int run = cta_scan32<TPR>(loc, &total, ws32);
-  for (int v = v0; v < v1; ++v) {
-    const uint4 x = ld(v);
-    uint4 o;
-    o.x = (unsigned)run; run += __popc(x.x);
-    o.y = (unsigned)run; run += __popc(x.y);
-    o.z = (unsigned)run; run += __popc(x.z);
-    o.w = (unsigned)run; run += __popc(x.w);
-    reinterpret_cast<uint4*>(pre)[v] = o;
-  }
-  return total;
-}
 
 
-template <typename VT>
+// SL2 > 0: level 2 (u32) and its prefix (u16) in shared memory, SL2 entries each (rows of at most
+// SL2 output entries: numeric group 10), else both in the per-CTA global slab (L2-resident).
+template <typename VT, int SL2>
 __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
   constexpr int TPR = 1024;
+  constexpr bool SH = SL2 > 0;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];
@@ -462,8 +473,10 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
   unsigned* l1 = reinterpret_cast<unsigned*>(smem_raw);
   unsigned* p1 = l1 + l1p;
   BlockFlat<VT, TPR, 2048>* bf = reinterpret_cast<BlockFlat<VT, TPR, 2048>*>(p1 + l1p);
-  unsigned* fine = reinterpret_cast<unsigned*>(static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride);
-  unsigned* pre2 = fine + a.slab_T;
+  unsigned* fine = SH ? reinterpret_cast<unsigned*>(reinterpret_cast<unsigned char*>(bf) + align16((int)sizeof(*bf)))
+                      : reinterpret_cast<unsigned*>(static_cast<unsigned char*>(a.slab) + (long long)blockIdx.x * a.slab_stride);
+  unsigned* pre2 = fine + (SH ? 0LL : a.slab_T);             // global: u32 prefix after level 2
+  uint16_t* pre2s = reinterpret_cast<uint16_t*>(fine + SL2);  // shared: u16 prefix (<= SL2 entries)
   const VT* __restrict__ av_g = static_cast<const VT*>(a.a_val);
   const VT* __restrict__ bv_g = static_cast<const VT*>(a.b_val);
   const int t = threadIdx.x;
@@ -498,7 +511,7 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
     });
     __syncthreads();
     const int nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
-    const bool ok = nb <= (int)a.slab_T;  // CTA-uniform; false only for inconsistent input
+    const bool ok = nb <= (SH ? SL2 : (int)a.slab_T);  // CTA-uniform; false only for inconsistent input
     if (ok) {
       uint4* f4 = reinterpret_cast<uint4*>(fine);
       for (int v = t; v < (nb + 3) >> 2; v += TPR) f4[v] = make_uint4(0u, 0u, 0u, 0u);
@@ -510,14 +523,20 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
         atomicOr(fine + blk_of(d), 1u << (d & 31));
       });
     __syncthreads();
-    const int n_total = ok ? prefix_popc32<TPR>(fine, nb, pre2, ws32[0], true) : 0;
+    int n_total = 0;
+    if (ok) {
+      if constexpr (SH) n_total = prefix_popc<TPR>(fine, nb, pre2s, ws32[0]);
+      else n_total = prefix_popc32<TPR>(fine, nb, pre2, ws32[0], true);
+    }
     if (t == 0 && n_total != cn) atomicOr(a.err_flags, 2);
     __syncthreads();
     if (ok && n_total == cn)
       walk([&](int k, VT v) {
         const unsigned d = (unsigned)(k - lo);
         const int b = blk_of(d);
-        const int r = (int)__ldcg(pre2 + b) + __popc(__ldcg(fine + b) & ((1u << (d & 31)) - 1u));
+        int r;
+        if constexpr (SH) r = (int)pre2s[b] + __popc(fine[b] & ((1u << (d & 31)) - 1u));
+        else r = (int)__ldcg(pre2 + b) + __popc(__ldcg(fine + b) & ((1u << (d & 31)) - 1u));
         atomicAdd(cv + r, v);
         cc[r] = k;
       });
@@ -525,13 +544,14 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
   }
 }
 
-template <typename VT>
+template <typename VT, int SL2>
 cudaError_t launch_rankbig_v(cudaStream_t s, const NumArgs& a, int grid) {
-  const int smem = rankbig_smem_bytes_v<VT>(a.l1_words);
+  const int smem = rankbig_smem_bytes_v<VT>(a.l1_words) + (SL2 > 0 ? align16((int)sizeof(BlockFlat<VT, 1024, 2048>)) -
+                                                                        (int)sizeof(BlockFlat<VT, 1024, 2048>) + 6 * SL2 : 0);
   static PerDevice configured;
-  cudaError_t e = prepare(k_num_rankbig<VT>, smem, configured);
+  cudaError_t e = prepare(k_num_rankbig<VT, SL2>, smem, configured);
   if (e != cudaSuccess) return e;
-  k_num_rankbig<VT><<<grid, 1024, smem, s>>>(a);
+  k_num_rankbig<VT, SL2><<<grid, 1024, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -572,13 +592,17 @@ cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const N
   return fp64 ? launch_rankacc_v<double>(s, group, a) : launch_rankacc_v<float>(s, group, a);
 }
 
-int rankbig_smem_bytes(bool fp64, int l1_words) {
-  return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_v<double>(l1_words) : rankbig_smem_bytes_v<float>(l1_words));
+int rankbig_smem_bytes(bool fp64, int l1_words, bool shared_l2) {
+  const int bfb = fp64 ? (int)sizeof(BlockFlat<double, 1024, 2048>) : (int)sizeof(BlockFlat<float, 1024, 2048>);
+  return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_v<double>(l1_words) : rankbig_smem_bytes_v<float>(l1_words)) +
+         (shared_l2 ? align16(bfb) - bfb + 6 * kRankBigSharedL2 : 0);
 }
 
-cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid) {
+cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, bool shared_l2) {
   if (a.nrows <= 0 || grid <= 0) return cudaSuccess;
-  return fp64 ? launch_rankbig_v<double>(s, a, grid) : launch_rankbig_v<float>(s, a, grid);
+  if (shared_l2)
+    return fp64 ? launch_rankbig_v<double, kRankBigSharedL2>(s, a, grid) : launch_rankbig_v<float, kRankBigSharedL2>(s, a, grid);
+  return fp64 ? launch_rankbig_v<double, 0>(s, a, grid) : launch_rankbig_v<float, 0>(s, a, grid);
 }
 
 cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a) {

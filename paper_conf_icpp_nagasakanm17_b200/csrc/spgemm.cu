@@ -118,6 +118,7 @@ struct spgemm_ctx {
   // symbolic optimistic-group rows counted exactly by the chunked rank-count kernel (R-MAT s22:
   // 1811 rows with n_prod_i > 16384)
   int rank_big_sym = 1;
+  int rank_big_shared = 1;  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
   bool small = false;    // the last symbolic call took the small-matrix path
   std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
@@ -632,6 +633,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->esc_pct = v; break;
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_BIG_SHARED: h->rank_big_shared = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_BIG_SYM:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_SYM must be 0, 1 or 2");
       h->rank_big_sym = (int)v; break;
@@ -1139,7 +1141,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
-                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->snap2.max_nnz,
+                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)h->snap2.max_nnz,
                                    na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words, (long long)h->wsort};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
@@ -1202,7 +1204,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             gc.slab_stride = bstride[c];
             gc.slab_T = (long long)kNumGroups[kNumCluster + c].upper;
             gc.l1_words = l1w_rank;
-            CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c]));
+            // group 10 (nnz_i <= 24576): level 2 in shared memory when it fits beside level 1
+            const bool shl2 = c == 0 && h->rank_big_shared && kNumGroups[kNumCluster].upper <= kRankBigSharedL2 &&
+                              rankbig_smem_bytes(fp64, l1w_rank, true) <= kSmemLimit;
+            CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c], shl2));
             h->gkind[1][g] = SPGEMM_KERNEL_RANK_BIG;
           } else {
             CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));

@@ -663,7 +663,8 @@ def test_rank_acc_big_rows(spg, dtype):
     A, B = _big_rows(31)
     A, B = A.with_values("uniform", 1), B.with_values("uniform", 2)
     got = check(spg, A, B, dtype, what="big rows rank")
-    assert sum(got[3]["num_rows"][10:13]) > 0, "no rows above the CTA groups"
+    assert got[3]["num_rows"][10] > 0 and sum(got[3]["num_rows"][11:13]) > 0, "no rows above the CTA groups"
+    check(spg, A, B, dtype, opts={"rank_big_shared": 0}, what="big rows rank, level 2 in global memory")
     check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
 
 
@@ -685,6 +686,24 @@ def test_rank_count_big_rows_chunked(spg, dtype):
     assert st["sym_overflow_rows"] == 0
     got = check(spg, A, B, dtype, opts={"rank_big_sym": 0}, what="big rows optimistic chain")
     assert got[3]["sym_kernel"][10] == 1 and got[3]["sym_overflow_rows"] > 0
+
+
+def test_rank_count_rows_above_65535_blocks(spg):
+    """Chunked big-row count on rows with more than 65535 non-empty 32-column blocks (n = 2^23:
+    the level-1 prefix needs 32 bits; R-MAT s23's heaviest rows)."""
+    rng = np.random.default_rng(34)
+    m, k, n = 6, 1 << 17, 1 << 23
+    la = rng.integers(4500, 5500, size=m)
+    rows = np.repeat(np.arange(m), la)
+    A = from_coo(m, k, rows, rng.integers(0, k, size=rows.size)).with_values("uniform", 1)
+    br = np.repeat(np.arange(k), 24)
+    B = from_coo(k, n, br, rng.integers(0, n, size=br.size)).with_values("uniform", 2)
+    blocks = [np.unique(B.col[np.concatenate([np.arange(B.rpt[q], B.rpt[q + 1])
+                                              for q in A.col[A.rpt[i]:A.rpt[i + 1]]])] >> 5).size
+              for i in range(A.m)]
+    assert min(blocks) > 65535, blocks
+    got = check(spg, A, B, np.float32, opts={"rank_big_sym": 2}, what="rows above 65535 blocks")
+    assert got[3]["sym_kernel"][10] == 2
 
 
 def test_rank_acc_big_rows_int_exact(spg):
