@@ -209,6 +209,12 @@ typedef enum {
                                        on the rank-big kernel keep the level-2 bitmap and its
                                        prefix in shared memory when they fit beside level 1
                                        (DESIGN.md §5.8); 0: in the per-CTA global slab */
+    SPGEMM_OPT_RANK_MID = 28,       /* numeric group 9 (4096 < nnz_i <= 8192) of the rank kernels
+                                       (DESIGN.md §5.8): 2 (default) products held in registers,
+                                       values reduced straight into the zeroed row of C at their
+                                       rank, 512-thread CTAs, two per SM; 1: persistent 512-thread
+                                       CTAs re-walking the products, level 2 in shared memory;
+                                       0: one 1024-thread CTA per row, the row kept in shared memory */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,

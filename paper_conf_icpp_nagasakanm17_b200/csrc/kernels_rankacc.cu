@@ -134,15 +134,18 @@ __device__ __forceinline__ void clear_words(unsigned* words, int W) {
 //   keys[UPPER] i32 (numeric) | fine[UPPER] u32 | bstart[KP*TPR/32+1] i32 | l1[L1W] u32 |
 //   pre2[UPPER] u16 (numeric) | p1[L1W] u16 (u32 for the chunked big-row count: more than
 //   65535 non-empty blocks)
-template <typename VT, bool NUM, int TPR, long long UPPER, int MC, int KP>
+// GOUT (numeric): no vals / keys arrays — values are reduced straight into the zeroed row of C
+// at their rank and keys stored there (two CTAs per SM fit; numeric group 9).
+template <typename VT, bool NUM, int TPR, long long UPPER, int MC, int KP, bool GOUT = false>
 struct RankLayout {
   static constexpr int ME = MC * TPR;  // metadata entries
+  static constexpr bool kOwnOut = NUM && !GOUT;
   static constexpr int kVals = 0;
-  static constexpr int kB0 = NUM ? align16((int)(UPPER * sizeof(VT))) : 0;
+  static constexpr int kB0 = kOwnOut ? align16((int)(UPPER * sizeof(VT))) : 0;
   static constexpr int kAv = kB0 + align16(ME * 8);
   static constexpr int kIncl = kAv + (NUM ? align16(ME * (int)sizeof(VT)) : 0);
   static constexpr int kKeys = kIncl + align16(ME * 4);
-  static constexpr int kFine = kKeys + (NUM ? align16((int)UPPER * 4) : 0);
+  static constexpr int kFine = kKeys + (kOwnOut ? align16((int)UPPER * 4) : 0);
   static constexpr int kBstart = kFine + align16((int)UPPER * 4);
   static constexpr int kL1 = kBstart + align16((KP * TPR / 32 + 1) * 4);
   static __host__ __device__ constexpr int pre2(int l1w) { return kL1 + align16(l1w * 4); }
@@ -182,10 +185,10 @@ struct SymView : SymArgs {
 };
 
 // One row, symbolic (NUM = false: writes nnz_i to c_cnt[row]) or numeric (writes the row of C).
-template <typename VT, bool NUM, int TPR, long long UPPER, int KP, int MC, typename Args>
+template <typename VT, bool NUM, int TPR, long long UPPER, int KP, int MC, bool GOUT = false, typename Args>
 __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* smem_raw, int (*ws32)[32],
                                          long long* ws64) {
-  using L = RankLayout<VT, NUM, TPR, UPPER, MC, KP>;
+  using L = RankLayout<VT, NUM, TPR, UPPER, MC, KP, GOUT>;
   constexpr int ME = L::ME;
   VT* vals = reinterpret_cast<VT*>(smem_raw + L::kVals);
   long long* sb0 = reinterpret_cast<long long*>(smem_raw + L::kB0);
@@ -263,12 +266,23 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
     const unsigned bit = 1u << (d & 31);
     if ((NUM || (unsigned)b < (unsigned)UPPER) && !(fine[b] & bit)) atomicOr(fine + b, bit);
   };
+  int32_t* cc_row = nullptr;
+  VT* cv_row = nullptr;
+  if constexpr (NUM && GOUT) {
+    cc_row = a.c_col + a.c_rpt[row];
+    cv_row = static_cast<VT*>(a.c_val) + a.c_rpt[row];
+  }
   auto accumulate = [&](int k, VT v) {
     const unsigned d = (unsigned)(k - lo);
     const int b = blk_of(d);
     const int r = (int)pre2[b] + __popc(fine[b] & ((1u << (d & 31)) - 1u));
-    atomicAdd(vals + r, v);
-    keys[r] = k;
+    if constexpr (GOUT) {
+      atomicAdd(cv_row + r, v);  // red.global.add into the zeroed row (working precision)
+      cc_row[r] = k;
+    } else {
+      atomicAdd(vals + r, v);
+      keys[r] = k;
+    }
   };
   BlockFlat<VT, TPR>* bf = reinterpret_cast<BlockFlat<VT, TPR>*>(sb0);
   static_assert(sizeof(BlockFlat<VT, TPR>) <= (size_t)(L::kKeys - L::kB0) + 16, "block-flat view");
@@ -337,7 +351,11 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
     const int n_total = ok ? prefix_popc<TPR>(fine, nb, pre2, ws32[0]) : 0;
     if (t == 0 && n_total != cn) atomicOr(a.err_flags, 2);
     const int nw = ok ? min(n_total, cn) : 0;
-    for (int r = t; r < nw; r += TPR) vals[r] = VT(0);
+    if constexpr (GOUT) {
+      for (int r = t; r < nw; r += TPR) cv_row[r] = VT(0);
+    } else {
+      for (int r = t; r < nw; r += TPR) vals[r] = VT(0);
+    }
     __syncthreads();
     // (vi) accumulate at the rank
     if (ok) {
@@ -351,17 +369,25 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
     }
     __syncthreads();
     // (vii) sorted, compact row -> C (coalesced)
-    int32_t* __restrict__ cc = a.c_col + c0;
-    VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
-    for (int r = t; r < nw; r += TPR) {
-      cc[r] = keys[r];
-      cv[r] = vals[r];
+    if constexpr (!GOUT) {
+      int32_t* __restrict__ cc = a.c_col + c0;
+      VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
+      for (int r = t; r < nw; r += TPR) {
+        cc[r] = keys[r];
+        cv[r] = vals[r];
+      }
     }
   }
 }
 
 template <typename VT>
 constexpr int rankbig_smem_bytes_v(int l1w) { return 2 * rankbig_l1pad_h(l1w) * 4 + (int)sizeof(BlockFlat<VT, 1024, 2048>); }
+// dynamic shared memory of k_num_rankbig<VT, SL2, TPR>
+template <typename VT, int SL2, int TPR>
+constexpr int rankbig_smem_bytes_t(int l1w) {
+  return 2 * rankbig_l1pad_h(l1w) * 4 + (SL2 > 0 ? align16((int)sizeof(BlockFlat<VT, TPR, 2048>)) + 6 * SL2
+                                                : (int)sizeof(BlockFlat<VT, TPR, 2048>));
+}
 
 // 40 registers (1536 threads per SM) for fp32 / symbolic; fp64 values need 64 (no spills)
 // (KP > 8 products per thread: 1280 threads, ~48 registers)
@@ -374,6 +400,17 @@ __global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT), KP>()) void k
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];
   rank_row<VT, true, TPR, UPPER, KP, MC>(static_cast<const NumView&>(a), a.rows[blockIdx.x], smem_raw, ws32, ws64);
+}
+
+// Numeric group 9 with the products in registers and the output reduced into C: TPR 512, two
+// CTAs per SM (the one-CTA-per-SM kernel idles the SM at every per-row barrier)
+template <typename VT, int TPR, long long UPPER, int KP, int MC>
+__global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankout(NumArgs a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ int ws32[2][32];
+  __shared__ long long ws64[33];
+  rank_row<VT, true, TPR, UPPER, KP, MC, true>(static_cast<const NumView&>(a), a.rows[blockIdx.x], smem_raw, ws32,
+                                               ws64);
 }
 
 template <int TPR, long long UPPER, int KP, int MC>
@@ -438,6 +475,19 @@ cudaError_t launch_rankcnt_big(cudaStream_t s, const SymArgs& a) {
   return cudaGetLastError();
 }
 
+constexpr RankCfg kRankOut9 = {512, 16, 2};
+template <typename VT>
+using RankOutL = RankLayout<VT, true, kRankOut9.TPR, 8192, kRankOut9.MC, kRankOut9.KP, true>;
+template <typename VT>
+cudaError_t launch_rankout_v(cudaStream_t s, const NumArgs& a) {
+  const int smem = RankOutL<VT>::bytes(a.l1_words);
+  static PerDevice configured;
+  cudaError_t e = prepare(k_num_rankout<VT, kRankOut9.TPR, 8192, kRankOut9.KP, kRankOut9.MC>, smem, configured);
+  if (e != cudaSuccess) return e;
+  k_num_rankout<VT, kRankOut9.TPR, 8192, kRankOut9.KP, kRankOut9.MC><<<(unsigned)a.nrows, kRankOut9.TPR, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
 template <typename VT>
 cudaError_t launch_rankacc_v(cudaStream_t s, int group, const NumArgs& a) {
   switch (group) {
@@ -460,10 +510,10 @@ cudaError_t launch_rankacc_v(cudaStream_t s, int group, const NumArgs& a) {
 
 
 // SL2 > 0: level 2 (u32) and its prefix (u16) in shared memory, SL2 entries each (rows of at most
-// SL2 output entries: numeric group 10), else both in the per-CTA global slab (L2-resident).
-template <typename VT, int SL2>
-__global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
-  constexpr int TPR = 1024;
+// SL2 output entries: numeric groups 9-10), else both in the per-CTA global slab (L2-resident).
+// TPR 512: two CTAs per SM (numeric group 9: one row's barriers no longer idle the SM).
+template <typename VT, int SL2, int TPR>
+__global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankbig(NumArgs a) {
   constexpr bool SH = SL2 > 0;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
@@ -544,14 +594,13 @@ __global__ __launch_bounds__(1024, 1) void k_num_rankbig(NumArgs a) {
   }
 }
 
-template <typename VT, int SL2>
+template <typename VT, int SL2, int TPR>
 cudaError_t launch_rankbig_v(cudaStream_t s, const NumArgs& a, int grid) {
-  const int smem = rankbig_smem_bytes_v<VT>(a.l1_words) + (SL2 > 0 ? align16((int)sizeof(BlockFlat<VT, 1024, 2048>)) -
-                                                                        (int)sizeof(BlockFlat<VT, 1024, 2048>) + 6 * SL2 : 0);
+  const int smem = rankbig_smem_bytes_t<VT, SL2, TPR>(a.l1_words);
   static PerDevice configured;
-  cudaError_t e = prepare(k_num_rankbig<VT, SL2>, smem, configured);
+  cudaError_t e = prepare(k_num_rankbig<VT, SL2, TPR>, smem, configured);
   if (e != cudaSuccess) return e;
-  k_num_rankbig<VT, SL2><<<grid, 1024, smem, s>>>(a);
+  k_num_rankbig<VT, SL2, TPR><<<grid, TPR, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -587,22 +636,40 @@ int rankcnt_smem_bytes(int group, int l1_words) {
   }
 }
 
+int rankout_smem_bytes(bool fp64, int l1_words) {
+  return kStaticRankBytes + (fp64 ? RankOutL<double>::bytes(l1_words) : RankOutL<float>::bytes(l1_words));
+}
+
+cudaError_t launch_numeric_rankout(cudaStream_t s, bool fp64, const NumArgs& a) {
+  if (a.nrows <= 0) return cudaSuccess;
+  return fp64 ? launch_rankout_v<double>(s, a) : launch_rankout_v<float>(s, a);
+}
+
 cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const NumArgs& a) {
   if (a.nrows <= 0) return cudaSuccess;
   return fp64 ? launch_rankacc_v<double>(s, group, a) : launch_rankacc_v<float>(s, group, a);
 }
 
-int rankbig_smem_bytes(bool fp64, int l1_words, bool shared_l2) {
-  const int bfb = fp64 ? (int)sizeof(BlockFlat<double, 1024, 2048>) : (int)sizeof(BlockFlat<float, 1024, 2048>);
-  return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_v<double>(l1_words) : rankbig_smem_bytes_v<float>(l1_words)) +
-         (shared_l2 ? align16(bfb) - bfb + 6 * kRankBigSharedL2 : 0);
+int rankbig_smem_bytes(bool fp64, int l1_words, int variant) {
+  switch (variant) {
+    case 1: return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_t<double, kRankBigSharedL2, 1024>(l1_words)
+                                            : rankbig_smem_bytes_t<float, kRankBigSharedL2, 1024>(l1_words));
+    case 2: return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_t<double, kRankMidSharedL2, 512>(l1_words)
+                                            : rankbig_smem_bytes_t<float, kRankMidSharedL2, 512>(l1_words));
+    default: return kStaticRankBytes + (fp64 ? rankbig_smem_bytes_t<double, 0, 1024>(l1_words)
+                                             : rankbig_smem_bytes_t<float, 0, 1024>(l1_words));
+  }
 }
 
-cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, bool shared_l2) {
+cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, int variant) {
   if (a.nrows <= 0 || grid <= 0) return cudaSuccess;
-  if (shared_l2)
-    return fp64 ? launch_rankbig_v<double, kRankBigSharedL2>(s, a, grid) : launch_rankbig_v<float, kRankBigSharedL2>(s, a, grid);
-  return fp64 ? launch_rankbig_v<double, 0>(s, a, grid) : launch_rankbig_v<float, 0>(s, a, grid);
+  switch (variant) {
+    case 1: return fp64 ? launch_rankbig_v<double, kRankBigSharedL2, 1024>(s, a, grid)
+                        : launch_rankbig_v<float, kRankBigSharedL2, 1024>(s, a, grid);
+    case 2: return fp64 ? launch_rankbig_v<double, kRankMidSharedL2, 512>(s, a, grid)
+                        : launch_rankbig_v<float, kRankMidSharedL2, 512>(s, a, grid);
+    default: return fp64 ? launch_rankbig_v<double, 0, 1024>(s, a, grid) : launch_rankbig_v<float, 0, 1024>(s, a, grid);
+  }
 }
 
 cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a) {

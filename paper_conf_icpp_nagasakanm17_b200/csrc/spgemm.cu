@@ -118,7 +118,11 @@ struct spgemm_ctx {
   // symbolic optimistic-group rows counted exactly by the chunked rank-count kernel (R-MAT s22:
   // 1811 rows with n_prod_i > 16384)
   int rank_big_sym = 1;
-  int rank_big_shared = 1;  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
+  int rank_big_shared = 1;
+  // numeric group 9: 2 = products in registers, output reduced into C, two 512-thread CTAs per SM
+  // (R-MAT s22 6.87 -> 5.54 ms); 1 = persistent rank-big kernel with level 2 in shared memory
+  // (6.32 ms); 0 = one 1024-thread CTA per row, the row in shared memory
+  int rank_mid = 2;  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
   bool small = false;    // the last symbolic call took the small-matrix path
   std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
@@ -634,6 +638,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_BIG_SHARED: h->rank_big_shared = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_MID:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_MID must be 0, 1 or 2");
+      h->rank_mid = (int)v; break;
     case SPGEMM_OPT_RANK_BIG_SYM:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_SYM must be 0, 1 or 2");
       h->rank_big_sym = (int)v; break;
@@ -1105,6 +1112,10 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const bool big_rank = h->rank_acc && h->rlohi.p != nullptr && h->num_min_group < 0 &&
                           rankbig_smem_bytes(fp64, l1w_rank) <= kSmemLimit;
     long long bstride[3] = {0, 0, 0}, bgrid[3] = {0, 0, 0}, btotal = 0;
+    // numeric group 9 on the persistent shared-memory rank kernel (RANK_MID)
+    const bool mid_rank = h->rank_mid == 1 && h->snap2.num_rows[kNumCluster - 1] > 0 && rank_acc_on(kNumCluster - 1) &&
+                          kNumGroups[kNumCluster - 1].upper <= kRankMidSharedL2 &&
+                          rankbig_smem_bytes(fp64, l1w_rank, 2) <= kSmemLimit / 2;
     for (int c = 0; c < 3; ++c) {
       const long long rows_c = (long long)h->snap2.num_rows[kNumCluster + c];
       if (rows_c == 0) continue;
@@ -1141,7 +1152,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
-                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)h->snap2.max_nnz,
+                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)mid_rank, (long long)h->rank_mid, (long long)h->snap2.max_nnz,
                                    na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words, (long long)h->wsort};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
@@ -1151,7 +1162,8 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                          (long long)h->rbits.p, (long long)h->perm1.p};
     const bool ge = group_events(h);
     auto enqueue = [&]() -> spgemm_status_t {
-      if (ctotal > 0 || btotal > 0) CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
+      if (ctotal > 0 || btotal > 0 || mid_rank)
+        CK(cudaMemsetAsync(dacc->row_counter, 0, sizeof(dacc->row_counter), h->stream));
       h->phase_streams = phase_concurrent(h, h->snap2.num_rows, kNumNumGroups);
       CK(fork(h));
       for (int g = 0; g < kNumNumGroups; ++g) {
@@ -1206,8 +1218,8 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             gc.l1_words = l1w_rank;
             // group 10 (nnz_i <= 24576): level 2 in shared memory when it fits beside level 1
             const bool shl2 = c == 0 && h->rank_big_shared && kNumGroups[kNumCluster].upper <= kRankBigSharedL2 &&
-                              rankbig_smem_bytes(fp64, l1w_rank, true) <= kSmemLimit;
-            CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c], shl2));
+                              rankbig_smem_bytes(fp64, l1w_rank, 1) <= kSmemLimit;
+            CK(launch_numeric_rankbig(st, fp64, gc, (int)bgrid[c], shl2 ? 1 : 0));
             h->gkind[1][g] = SPGEMM_KERNEL_RANK_BIG;
           } else {
             CK(launch_numeric_cluster(st, fp64, 2 << c, gc, nullptr));
@@ -1233,6 +1245,20 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
           if (h->tiny && h->num_min_group < 0 && g <= 1) {
             CK(launch_numeric_tiny(st, g, fp64, ga));
             h->gkind[1][g] = SPGEMM_KERNEL_TINY;
+          } else if (rank_acc_on(g) && g == kNumCluster - 1 && h->rank_mid == 2 &&
+                     rankout_smem_bytes(fp64, l1w_rank) <= kSmemLimit / 2) {
+            NumArgs ra = ga;
+            ra.l1_words = l1w_rank;
+            CK(launch_numeric_rankout(st, fp64, ra));
+            h->gkind[1][g] = SPGEMM_KERNEL_RANK;
+          } else if (rank_acc_on(g) && g == kNumCluster - 1 && mid_rank) {
+            // group 9: persistent rank kernel, two 512-thread CTAs per SM, level 2 in shared
+            // memory, values reduced into C
+            NumArgs ra = ga;
+            ra.l1_words = l1w_rank;
+            ra.row_counter = dacc->row_counter + 3;
+            CK(launch_numeric_rankbig(st, fp64, ra, (int)std::min<long long>(rows, 2LL * h->num_sms), 2));
+            h->gkind[1][g] = SPGEMM_KERNEL_RANK_BIG;
           } else if (rank_acc_on(g)) {
             NumArgs ra = ga;
             ra.l1_words = l1w_rank;

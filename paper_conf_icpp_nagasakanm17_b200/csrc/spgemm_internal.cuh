@@ -846,17 +846,24 @@ cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const N
 int rankacc_smem_bytes(int group, bool fp64, int l1_words);
 cudaError_t launch_symbolic_rankcnt(cudaStream_t s, int group, const SymArgs& a);
 int rankcnt_smem_bytes(int group, int l1_words);
-// shared_l2: the level-2 bitmap and its prefix in shared memory (rows of <= kRankBigSharedL2
-// output entries, numeric group 10), else in the per-CTA global slab
+// Rank-big kernel variants: 0 = level-2 bitmap and prefix in a per-CTA global slab (1024 threads);
+// 1 = in shared memory, rows of <= kRankBigSharedL2 output entries (numeric group 10, 1024
+// threads); 2 = in shared memory, rows of <= kRankMidSharedL2 entries (numeric group 9, 512
+// threads, two CTAs per SM)
 constexpr int kRankBigSharedL2 = 24576;
-cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, bool shared_l2);
+constexpr int kRankMidSharedL2 = 8192;
+cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, int variant);
+// numeric group 9: products in registers, output reduced into C (no vals / keys arrays), 512 threads,
+// two CTAs per SM
+cudaError_t launch_numeric_rankout(cudaStream_t s, bool fp64, const NumArgs& a);
+int rankout_smem_bytes(bool fp64, int l1_words);
 cudaError_t launch_symbolic_tiny(cudaStream_t s, int group, const SymArgs& a);
 cudaError_t launch_small_symbolic(cudaStream_t s, long long m, long long k, const int64_t* a_rpt, const int32_t* a_col,
                                   const int64_t* b_rpt, const int32_t* b_col, int64_t* c_cnt, int64_t* nprod,
                                   DevAcc* acc);
 cudaError_t launch_small_numeric(cudaStream_t s, bool fp64, const NumArgs& a, long long m);
 cudaError_t launch_numeric_tiny(cudaStream_t s, int group, bool fp64, const NumArgs& a);
-int rankbig_smem_bytes(bool fp64, int l1_words, bool shared_l2 = false);
+int rankbig_smem_bytes(bool fp64, int l1_words, int variant = 0);
 cudaError_t launch_symbolic_cluster(cudaStream_t s, const SymArgs& a, const int32_t* rows, const int* count,
                                     int32_t* overflow2, int* count2, int fill_limit, int max_rows);
 cudaError_t launch_numeric_cluster(cudaStream_t s, bool fp64, int cs, const NumArgs& a, int* nclusters_out);

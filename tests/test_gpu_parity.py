@@ -665,6 +665,7 @@ def test_rank_acc_big_rows(spg, dtype):
     got = check(spg, A, B, dtype, what="big rows rank")
     assert got[3]["num_rows"][10] > 0 and sum(got[3]["num_rows"][11:13]) > 0, "no rows above the CTA groups"
     check(spg, A, B, dtype, opts={"rank_big_shared": 0}, what="big rows rank, level 2 in global memory")
+    check(spg, A, B, dtype, opts={"rank_mid": 0}, what="big rows rank, group 9 one CTA per row")
     check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
 
 
@@ -704,6 +705,26 @@ def test_rank_count_rows_above_65535_blocks(spg):
     assert min(blocks) > 65535, blocks
     got = check(spg, A, B, np.float32, opts={"rank_big_sym": 2}, what="rows above 65535 blocks")
     assert got[3]["sym_kernel"][10] == 2
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_rank_mid_group9_rows(spg, dtype):
+    """Numeric group 9 (4096 < nnz_i <= 8192): products in registers, output reduced into C,
+    two CTAs per SM (RANK_MID 2, default); the persistent rank-big variant (1) and one CTA per row
+    with the row in shared memory (0); all against the oracle."""
+    rng = np.random.default_rng(35)
+    m, k, n = 500, 1 << 17, 1 << 21
+    la = rng.integers(180, 340, size=m)
+    rows = np.repeat(np.arange(m), la)
+    A = from_coo(m, k, rows, rng.integers(0, k, size=rows.size)).with_values("uniform", 1)
+    br = np.repeat(np.arange(k), 24)
+    B = from_coo(k, n, br, rng.integers(0, n, size=br.size)).with_values("uniform", 2)
+    got = check(spg, A, B, dtype, what="group 9 registers, output reduced into C")
+    assert got[3]["num_rows"][9] > 0 and got[3]["num_kernel"][9] == 2, (got[3]["num_rows"][9], got[3]["num_kernel"])
+    got = check(spg, A, B, dtype, opts={"rank_mid": 1}, what="group 9 persistent rank-big")
+    assert got[3]["num_kernel"][9] == 6
+    got = check(spg, A, B, dtype, opts={"rank_mid": 0}, what="group 9 one CTA per row")
+    assert got[3]["num_kernel"][9] == 2
 
 
 def test_rank_acc_big_rows_int_exact(spg):
