@@ -215,6 +215,9 @@ typedef enum {
                                        rank, 512-thread CTAs, two per SM; 1: persistent 512-thread
                                        CTAs re-walking the products, level 2 in shared memory;
                                        0: one 1024-thread CTA per row, the row kept in shared memory */
+    SPGEMM_OPT_RANK_GOUT = 29,      /* 1: numeric rank groups 3-8 reduce values straight into the
+                                       zeroed row of C at their rank instead of a shared-memory
+                                       row (less shared memory per CTA).  Default 0 */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,

@@ -405,7 +405,7 @@ __global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT), KP>()) void k
 // Numeric group 9 with the products in registers and the output reduced into C: TPR 512, two
 // CTAs per SM (the one-CTA-per-SM kernel idles the SM at every per-row barrier)
 template <typename VT, int TPR, long long UPPER, int KP, int MC>
-__global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankout(NumArgs a) {
+__global__ __launch_bounds__(TPR, rank_min_blocks<TPR, sizeof(VT), KP>()) void k_num_rankout(NumArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ int ws32[2][32];
   __shared__ long long ws64[33];
@@ -475,16 +475,19 @@ cudaError_t launch_rankcnt_big(cudaStream_t s, const SymArgs& a) {
   return cudaGetLastError();
 }
 
-constexpr RankCfg kRankOut9 = {512, 16, 2};
-template <typename VT>
-using RankOutL = RankLayout<VT, true, kRankOut9.TPR, 8192, kRankOut9.MC, kRankOut9.KP, true>;
-template <typename VT>
-cudaError_t launch_rankout_v(cudaStream_t s, const NumArgs& a) {
-  const int smem = RankOutL<VT>::bytes(a.l1_words);
+// output-in-C rank kernels: group 9 at 512 threads (two CTAs per SM), groups 3-8 at kRankNum
+constexpr RankCfg rank_out_cfg(int g) { return g == 9 ? RankCfg{512, 16, 2} : kRankNum[g]; }
+template <typename VT, int G>
+using RankOutL = RankLayout<VT, true, rank_out_cfg(G).TPR, kNumGroups[G].upper, rank_out_cfg(G).MC, rank_out_cfg(G).KP, true>;
+template <typename VT, int G>
+cudaError_t launch_rankout_k(cudaStream_t s, const NumArgs& a) {
+  constexpr RankCfg c = rank_out_cfg(G);
+  constexpr long long UPPER = kNumGroups[G].upper;
+  const int smem = RankOutL<VT, G>::bytes(a.l1_words);
   static PerDevice configured;
-  cudaError_t e = prepare(k_num_rankout<VT, kRankOut9.TPR, 8192, kRankOut9.KP, kRankOut9.MC>, smem, configured);
+  cudaError_t e = prepare(k_num_rankout<VT, c.TPR, UPPER, c.KP, c.MC>, smem, configured);
   if (e != cudaSuccess) return e;
-  k_num_rankout<VT, kRankOut9.TPR, 8192, kRankOut9.KP, kRankOut9.MC><<<(unsigned)a.nrows, kRankOut9.TPR, smem, s>>>(a);
+  k_num_rankout<VT, c.TPR, UPPER, c.KP, c.MC><<<(unsigned)a.nrows, c.TPR, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -636,13 +639,25 @@ int rankcnt_smem_bytes(int group, int l1_words) {
   }
 }
 
-int rankout_smem_bytes(bool fp64, int l1_words) {
-  return kStaticRankBytes + (fp64 ? RankOutL<double>::bytes(l1_words) : RankOutL<float>::bytes(l1_words));
+int rankout_smem_bytes(int group, bool fp64, int l1_words) {
+  switch (group) {
+#define SPG_G(I) \
+  case I: return kStaticRankBytes + (fp64 ? RankOutL<double, I>::bytes(l1_words) : RankOutL<float, I>::bytes(l1_words));
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#undef SPG_G
+    default: return INT_MAX;
+  }
 }
 
-cudaError_t launch_numeric_rankout(cudaStream_t s, bool fp64, const NumArgs& a) {
+cudaError_t launch_numeric_rankout(cudaStream_t s, int group, bool fp64, const NumArgs& a) {
   if (a.nrows <= 0) return cudaSuccess;
-  return fp64 ? launch_rankout_v<double>(s, a) : launch_rankout_v<float>(s, a);
+  switch (group) {
+#define SPG_G(I) \
+  case I: return fp64 ? launch_rankout_k<double, I>(s, a) : launch_rankout_k<float, I>(s, a);
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+#undef SPG_G
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 cudaError_t launch_numeric_rankacc(cudaStream_t s, int group, bool fp64, const NumArgs& a) {

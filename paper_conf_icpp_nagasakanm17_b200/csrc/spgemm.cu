@@ -122,7 +122,8 @@ struct spgemm_ctx {
   // numeric group 9: 2 = products in registers, output reduced into C, two 512-thread CTAs per SM
   // (R-MAT s22 6.87 -> 5.54 ms); 1 = persistent rank-big kernel with level 2 in shared memory
   // (6.32 ms); 0 = one 1024-thread CTA per row, the row in shared memory
-  int rank_mid = 2;  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
+  int rank_mid = 2;
+  int rank_gout = 0;  // numeric rank groups 3-8 with the output reduced into C (no vals/keys arrays)  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
   bool small = false;    // the last symbolic call took the small-matrix path
   std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
@@ -638,6 +639,7 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_BIG_SHARED: h->rank_big_shared = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_GOUT: h->rank_gout = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_MID:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_MID must be 0, 1 or 2");
       h->rank_mid = (int)v; break;
@@ -1152,7 +1154,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
-                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)mid_rank, (long long)h->rank_mid, (long long)h->snap2.max_nnz,
+                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)mid_rank, (long long)h->rank_mid, (long long)h->rank_gout, (long long)h->snap2.max_nnz,
                                    na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words, (long long)h->wsort};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
@@ -1245,11 +1247,11 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
           if (h->tiny && h->num_min_group < 0 && g <= 1) {
             CK(launch_numeric_tiny(st, g, fp64, ga));
             h->gkind[1][g] = SPGEMM_KERNEL_TINY;
-          } else if (rank_acc_on(g) && g == kNumCluster - 1 && h->rank_mid == 2 &&
-                     rankout_smem_bytes(fp64, l1w_rank) <= kSmemLimit / 2) {
+          } else if (rank_acc_on(g) && ((g == kNumCluster - 1 && h->rank_mid == 2) || (g < kNumCluster - 1 && h->rank_gout)) &&
+                     rankout_smem_bytes(g, fp64, l1w_rank) <= (g == kNumCluster - 1 ? kSmemLimit / 2 : kSmemLimit)) {
             NumArgs ra = ga;
             ra.l1_words = l1w_rank;
-            CK(launch_numeric_rankout(st, fp64, ra));
+            CK(launch_numeric_rankout(st, g, fp64, ra));
             h->gkind[1][g] = SPGEMM_KERNEL_RANK;
           } else if (rank_acc_on(g) && g == kNumCluster - 1 && mid_rank) {
             // group 9: persistent rank kernel, two 512-thread CTAs per SM, level 2 in shared

@@ -853,10 +853,10 @@ int rankcnt_smem_bytes(int group, int l1_words);
 constexpr int kRankBigSharedL2 = 24576;
 constexpr int kRankMidSharedL2 = 8192;
 cudaError_t launch_numeric_rankbig(cudaStream_t s, bool fp64, const NumArgs& a, int grid, int variant);
-// numeric group 9: products in registers, output reduced into C (no vals / keys arrays), 512 threads,
-// two CTAs per SM
-cudaError_t launch_numeric_rankout(cudaStream_t s, bool fp64, const NumArgs& a);
-int rankout_smem_bytes(bool fp64, int l1_words);
+// rank kernels with the output reduced straight into C (no vals / keys arrays in shared memory):
+// numeric group 9 at 512 threads, two CTAs per SM; groups 3-8 at their kRankNum shapes
+cudaError_t launch_numeric_rankout(cudaStream_t s, int group, bool fp64, const NumArgs& a);
+int rankout_smem_bytes(int group, bool fp64, int l1_words);
 cudaError_t launch_symbolic_tiny(cudaStream_t s, int group, const SymArgs& a);
 cudaError_t launch_small_symbolic(cudaStream_t s, long long m, long long k, const int64_t* a_rpt, const int32_t* a_col,
                                   const int64_t* b_rpt, const int32_t* b_col, int64_t* c_cnt, int64_t* nprod,

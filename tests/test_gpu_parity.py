@@ -727,6 +727,14 @@ def test_rank_mid_group9_rows(spg, dtype):
     assert got[3]["num_kernel"][9] == 2
 
 
+@pytest.mark.parametrize("name", ["rmat14", "webbase_small"])
+def test_rank_gout_groups(spg, name):
+    """RANK_GOUT: rank groups 3-8 reduce into the row of C instead of a shared-memory row."""
+    A = _mixed_small() if name == "webbase_small" else synth.rmat(14).with_values("uniform", 9)
+    got = check(spg, A, A, np.float32, opts={"rank_gout": 1}, what=f"{name} rank_gout")
+    assert _rank_rows(got[3]) > 0
+
+
 def test_rank_acc_big_rows_int_exact(spg):
     A, B = _big_rows(32)
     check(spg, A.with_values("int", 3), B.with_values("int", 4), np.float32, exact=True, what="big rows int")
