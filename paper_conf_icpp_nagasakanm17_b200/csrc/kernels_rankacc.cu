@@ -357,8 +357,9 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
       for (int r = t; r < nw; r += TPR) vals[r] = VT(0);
     }
     __syncthreads();
-    // (vi) accumulate at the rank
-    if (ok) {
+    // (vi) accumulate at the rank (GOUT writes C directly: only when the counts agree, so an
+    // inconsistent input cannot write past the row; err_flags bit 1 is raised above)
+    if (ok && (!GOUT || n_total == cn)) {
       if (fast) {
 #pragma unroll
         for (int u = 0; u < KP; ++u)
