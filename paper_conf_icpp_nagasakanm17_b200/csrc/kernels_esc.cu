@@ -327,13 +327,16 @@ __device__ __forceinline__ int esc_scan_counts(int* c, int* ws, int (&vals)[N]) 
   return tot;
 }
 
+#ifndef SPG_ESC64_OCC
+#define SPG_ESC64_OCC 1280  // fp64 threads per SM (R-MAT s22 fp64: 1024 / MC 2 71.9 ms, 1280 / MC 1 67.5, 1536 75.5)
+#endif
 #ifndef SPG_ESC_OCC
 #define SPG_ESC_OCC 1536
 #endif
 constexpr int kEscOcc = SPG_ESC_OCC;  // fp32 threads per SM the launch bounds ask for
 
 template <typename VT, int TPR, int KP, int MC, int R>
-__global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? 1024 : kEscOcc) / TPR) void k_num_esc(NumArgs a) {
+__global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? SPG_ESC64_OCC : kEscOcc) / TPR) void k_num_esc(NumArgs a) {
   using S = NumEscSmem<VT, TPR, KP, MC, R>;
   constexpr int CAP = S::CAP;
   static_assert(CAP <= 4096, "bucket starts and output bases are packed into 16 and 15 bits");
@@ -622,8 +625,23 @@ constexpr EscCfg kEscNum32[] = {{0, 0, 0},
                                 {512 * 8 / kEscKp, kEscKp, SPG_ESC_MC},
                                 {1024, 8, 2},
                                 {1024, 16, 1}};
-constexpr EscCfg kEscNum64[] = {{0, 0, 0},  {0, 0, 0},  {256, 8, 2},  {256, 8, 2},  {256, 8, 2},
-                                {256, 8, 2},  {256, 8, 2},  {512, 8, 2},  {1024, 8, 2}, {1024, 16, 1}};
+#ifndef SPG_ESC64_TPR
+#define SPG_ESC64_TPR 256
+#endif
+#ifndef SPG_ESC64_MC
+#define SPG_ESC64_MC 1
+#endif
+constexpr int kEsc64Tpr = SPG_ESC64_TPR;  // fp64 groups 2-5 (group 6: max(256, this))
+constexpr EscCfg kEscNum64[] = {{0, 0, 0},
+                                {0, 0, 0},
+                                {kEsc64Tpr, 8, SPG_ESC64_MC},
+                                {kEsc64Tpr, 8, SPG_ESC64_MC},
+                                {kEsc64Tpr, 8, SPG_ESC64_MC},
+                                {kEsc64Tpr >= 128 ? kEsc64Tpr : 128, 8, SPG_ESC64_MC},
+                                {256, 8, SPG_ESC64_MC},
+                                {512, 8, SPG_ESC64_MC},
+                                {1024, 8, 2},
+                                {1024, 16, 1}};
 template <typename VT>
 constexpr EscCfg esc_num_cfg(int g) { return sizeof(VT) == 8 ? kEscNum64[g] : kEscNum32[g]; }
 

@@ -9,8 +9,9 @@ import torch
 import synth
 import paper_conf_icpp_nagasakanm17_b200 as P
 
-A = synth.config(sys.argv[1], "uniform", 7).astype(np.float32)
-dA = P.CsrMatrix.from_host(A, "cuda", torch.float32)
+F64 = os.environ.get("GT_DTYPE") == "f64"
+A = synth.config(sys.argv[1], "uniform", 7).astype(np.float64 if F64 else np.float32)
+dA = P.CsrMatrix.from_host(A, "cuda", torch.float64 if F64 else torch.float32)
 with P.Handle() as h:
     h.set_option("timing", 2).set_option("streams", 0)
     for kv in sys.argv[2:]:
