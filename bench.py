@@ -176,6 +176,13 @@ def load_traffic(config, dtype, phase, g):
     return (e["dram_bytes"], e["source"]) if e else (None, None)
 
 
+def load_inst(config, dtype, phase, g):
+    """Executed warp instructions and issue-active % of this group's launch (same ncu capture)."""
+    p = os.path.join(ROOT, "profiles", "traffic_r02.json")
+    e = json.load(open(p)).get(f"{config}|{dtype}|{phase}|g{g}") if os.path.exists(p) else None
+    return (e.get("warp_inst"), e.get("issue_active_pct")) if e else (None, None)
+
+
 # ----------------------------------------------------------------------------- reference arm
 def reference_sample(A, nprod_rows, frac):
     """Rows [0, r) of A holding about `frac` of the intermediate products (hubs included)."""
@@ -365,6 +372,18 @@ def run_ours(args):
                 "attribution": "per-group CUDA events, group kernels serialised on one stream (one extra step)",
                 "top_groups": [{"phase": p, "group": q, "kernel": (SYM_KERNEL if p == "sym" else NUM_KERNEL).get(k, "?"),
                                 "ms": m} for m, p, q, k in groups[:6]]}
+    # the roof that binds the graph kernels: instruction issue — executed warp
+    # instructions of the same launch (ncu) / kernel time against 4 issue slots per SM per cycle
+    winst, issue_pct = load_inst(args.config, args.dtype, ph, g)
+    if winst:
+        sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        peak_issue = sms * 4 * 1965e6 / 1e9  # G warp-instructions/s at the B200's max SM clock
+        ach_issue = winst / (k_ms / 1e3) / 1e9
+        roofline["issue"] = {"bound": "issue", "achieved": ach_issue, "peak": peak_issue,
+                             "unit": "G warp-instr/s", "frac": ach_issue / peak_issue,
+                             "ncu_issue_active_pct": issue_pct, "warp_inst_per_launch": int(winst),
+                             "peak_source": f"{sms} SMs x 4 schedulers x 1965 MHz (max SM clock, nvidia-smi)",
+                             "source": "ncu smsp__inst_executed.sum of the same launch (scripts/traffic.py)"}
 
     # measured peak device memory of one step (all library workspace through torch's allocator)
     peak_mem = None

@@ -3,6 +3,8 @@ roofline.traffic (profiles/traffic_r02.json; run on the GPU box).
 
     python scripts/traffic.py CONFIG [DTYPE] [--top N]
 
+(round 2: also executed warp instructions and issue-active %, for the issue roofline)
+
 1. runs one serialised multiply (streams 0, per-group events) and lists the groups with their
    kernel family and time (same as bench.py's attribution step);
 2. for each of the N slowest groups runs ncu on one more serialised multiply restricted to the
@@ -66,7 +68,8 @@ def main():
         done.add(kname)
         # all groups of this family, in launch order
         fam_groups = sorted(q for _, p, q, k in groups if k == kname and p == ph)
-        r = subprocess.run(["ncu", "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
+        r = subprocess.run(["ncu", "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,"
+                            "smsp__inst_executed.sum,smsp__issue_active.avg.pct_of_peak_sustained_active",
                             "--clock-control", "none", "--csv", "--print-units", "base", "-k", f"regex:{kname}",
                             sys.executable, __file__, "--child", config, dtype], capture_output=True, text=True)
         rows = list(csv.reader(io.StringIO(r.stdout)))
@@ -86,6 +89,9 @@ def main():
             m = launches[i]
             byts = int(m.get("dram__bytes_read.sum", 0) + m.get("dram__bytes_write.sum", 0))
             db[f"{config}|{dtype}|{ph}|g{q}"] = {"dram_bytes": byts, "ncu_time_ns": m.get("gpu__time_duration.sum"),
+                                                 "warp_inst": int(m.get("smsp__inst_executed.sum", 0)),
+                                                 "issue_active_pct": m.get(
+                                                     "smsp__issue_active.avg.pct_of_peak_sustained_active"),
                                                  "kernel": kname,
                                                  "source": f"ncu --metrics dram__bytes_read/write.sum, serialised "
                                                            f"multiply of {config} {dtype} (scripts/traffic.py)"}
