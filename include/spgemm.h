@@ -208,7 +208,9 @@ typedef enum {
     SPGEMM_OPT_RANK_BIG_SHARED = 27,/* 1 (default): numeric rows of group 10 (8192 < nnz_i <= 24576)
                                        on the rank-big kernel keep the level-2 bitmap and its
                                        prefix in shared memory when they fit beside level 1
-                                       (DESIGN.md §5.8); 0: in the per-CTA global slab */
+                                       (DESIGN.md §5.8); 0: in the per-CTA global slab; 2: one
+                                       1024-thread CTA per row with the products in registers and
+                                       the output reduced into C (measured equal at R-MAT s22) */
     SPGEMM_OPT_RANK_MID = 28,       /* numeric group 9 (4096 < nnz_i <= 8192) of the rank kernels
                                        (DESIGN.md §5.8): 2 (default) products held in registers,
                                        values reduced straight into the zeroed row of C at their

@@ -477,7 +477,9 @@ cudaError_t launch_rankcnt_big(cudaStream_t s, const SymArgs& a) {
 }
 
 // output-in-C rank kernels: group 9 at 512 threads (two CTAs per SM), groups 3-8 at kRankNum
-constexpr RankCfg rank_out_cfg(int g) { return g == 9 ? RankCfg{512, 16, 2} : kRankNum[g]; }
+constexpr RankCfg rank_out_cfg(int g) {
+  return g == 10 ? RankCfg{1024, 16, 2} : g == 9 ? RankCfg{512, 16, 2} : kRankNum[g];
+}
 template <typename VT, int G>
 using RankOutL = RankLayout<VT, true, rank_out_cfg(G).TPR, kNumGroups[G].upper, rank_out_cfg(G).MC, rank_out_cfg(G).KP, true>;
 template <typename VT, int G>
@@ -644,7 +646,7 @@ int rankout_smem_bytes(int group, bool fp64, int l1_words) {
   switch (group) {
 #define SPG_G(I) \
   case I: return kStaticRankBytes + (fp64 ? RankOutL<double, I>::bytes(l1_words) : RankOutL<float, I>::bytes(l1_words));
-    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9) SPG_G(10)
 #undef SPG_G
     default: return INT_MAX;
   }
@@ -655,7 +657,7 @@ cudaError_t launch_numeric_rankout(cudaStream_t s, int group, bool fp64, const N
   switch (group) {
 #define SPG_G(I) \
   case I: return fp64 ? launch_rankout_k<double, I>(s, a) : launch_rankout_k<float, I>(s, a);
-    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9)
+    SPG_G(3) SPG_G(4) SPG_G(5) SPG_G(6) SPG_G(7) SPG_G(8) SPG_G(9) SPG_G(10)
 #undef SPG_G
     default: return cudaErrorInvalidValue;
   }

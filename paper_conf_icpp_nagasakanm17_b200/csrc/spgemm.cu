@@ -638,7 +638,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       h->esc_pct = v; break;
     case SPGEMM_OPT_ESC_GROUPS: h->esc_mask = v; break;
     case SPGEMM_OPT_SMALL: h->small_opt = v ? 1 : 0; break;
-    case SPGEMM_OPT_RANK_BIG_SHARED: h->rank_big_shared = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_BIG_SHARED:
+      if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_SHARED must be 0, 1 or 2");
+      h->rank_big_shared = (int)v; break;
     case SPGEMM_OPT_RANK_GOUT: h->rank_gout = v ? 1 : 0; break;
     case SPGEMM_OPT_RANK_MID:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_MID must be 0, 1 or 2");
@@ -1211,7 +1213,13 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(cudaMalloc(&gc.prof, sizeof(unsigned long long) * 4 * rows));
             CK(cudaMemset(gc.prof, 0, sizeof(unsigned long long) * 4 * rows));
           }
-          if (big_rank) {
+          if (big_rank && c == 0 && h->rank_big_shared == 2 && rankout_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit) {
+            // group 10: products in registers, output reduced into C, one 1024-thread CTA per row
+            NumArgs ro = ga;
+            ro.l1_words = l1w_rank;
+            CK(launch_numeric_rankout(st, g, fp64, ro));
+            h->gkind[1][g] = SPGEMM_KERNEL_RANK;
+          } else if (big_rank) {
             long long boff = 0;
             for (int q = 0; q < c; ++q) boff += bgrid[q] * bstride[q];
             gc.slab = static_cast<unsigned char*>(h->num_slab_c.p) + boff;

@@ -665,6 +665,7 @@ def test_rank_acc_big_rows(spg, dtype):
     got = check(spg, A, B, dtype, what="big rows rank")
     assert got[3]["num_rows"][10] > 0 and sum(got[3]["num_rows"][11:13]) > 0, "no rows above the CTA groups"
     check(spg, A, B, dtype, opts={"rank_big_shared": 0}, what="big rows rank, level 2 in global memory")
+    check(spg, A, B, dtype, opts={"rank_big_shared": 2}, what="big rows rank, group 10 in registers, output in C")
     check(spg, A, B, dtype, opts={"rank_mid": 0}, what="big rows rank, group 9 one CTA per row")
     check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
 
