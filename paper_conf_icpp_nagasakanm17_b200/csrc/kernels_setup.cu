@@ -523,8 +523,11 @@ __global__ __launch_bounds__(kSetupThreads) void k_scan_down(long long m, int64_
 // three; chunks of 4096 staged through shared memory with coalesced loads and stores, a running
 // carry across chunks.
 constexpr int kSmallScanChunk = 4096;
+// host_acc != nullptr: afterwards the CTA copies the whole DevAcc `acc` (the total included) to
+// host_acc, pinned host memory the kernel writes through PCIe (no separate D2H copy node).
 __global__ __launch_bounds__(1024) void k_scan_small(long long m, int64_t* __restrict__ x,
-                                                     long long* __restrict__ total_out) {
+                                                     long long* __restrict__ total_out, const DevAcc* acc,
+                                                     DevAcc* host_acc) {
   __shared__ long long tile[kSmallScanChunk];
   __shared__ long long ws[33];
   constexpr int PER = kSmallScanChunk / 1024;
@@ -559,6 +562,13 @@ __global__ __launch_bounds__(1024) void k_scan_small(long long m, int64_t* __res
     __syncthreads();
   }
   if (threadIdx.x == 0 && total_out) *total_out = carry;
+  if (host_acc) {
+    __syncthreads();  // the total above, the counters of the previous kernels
+    static_assert(sizeof(DevAcc) % 4 == 0, "DevAcc words");
+    const unsigned* src = reinterpret_cast<const unsigned*>(acc);
+    unsigned* dst = reinterpret_cast<unsigned*>(host_acc);
+    for (int i = threadIdx.x; i < (int)(sizeof(DevAcc) / 4); i += 1024) dst[i] = src[i];
+  }
 }
 
 // ------------------------------------------------------------------ validation
@@ -677,9 +687,9 @@ cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, c
   return scan_inclusive(s, m, c_rpt + 1, grp1, grp2, acc, b, esc, tile_ws, &acc->nnzc, nlaunch);
 }
 
-cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc) {
+cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc, DevAcc* host_acc) {
   if (m <= 0) return cudaSuccess;
-  k_scan_small<<<1, 1024, 0, s>>>(m, c_rpt + 1, &acc->nnzc);
+  k_scan_small<<<1, 1024, 0, s>>>(m, c_rpt + 1, &acc->nnzc, acc, host_acc);
   return cudaGetLastError();
 }
 

@@ -156,6 +156,7 @@ struct spgemm_ctx {
   bool perm2_ready = false;
   bool group_sums_done = false;  // per-group n_prod/nnz sums (computed on demand by get_stats)
   DevAcc* hacc = nullptr;      // pinned
+  DevAcc* hacc_dev = nullptr;  // the same memory as a device pointer (mapped pinned memory)
   long long* hends = nullptr;  // pinned: a_rpt[0], a_rpt[m], b_rpt[0], b_rpt[k]
   DevAcc snap1{}, snap2{};
   spgemm_stats_t stats{};
@@ -537,6 +538,7 @@ spgemm_status_t spgemm_create(spgemm_handle_t* out, int device, void* stream, co
     }
   }
   if (e == cudaSuccess) e = cudaMallocHost(&h->hacc, sizeof(DevAcc));
+  if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->hacc_dev), h->hacc, 0);
   if (e == cudaSuccess) e = cudaMallocHost(&h->hends, 4 * sizeof(long long));
   *out = h;
   if (e != cudaSuccess) return fail_cuda(h, e, "spgemm_create");
@@ -740,8 +742,8 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
       CK(cudaMemsetAsync(h->acc.p, 0, sizeof(DevAcc), h->stream));
       CK(launch_small_symbolic(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, c_rpt + 1,
                                static_cast<int64_t*>(h->nprod.p), dacc));
-      CK(launch_scan_small(h->stream, m, c_rpt, dacc));
-      CK(cudaMemcpyAsync(h->hacc, dacc, sizeof(DevAcc), cudaMemcpyDeviceToHost, h->stream));
+      // the scan kernel writes the counters straight to the pinned host copy (one graph node less)
+      CK(launch_scan_small(h->stream, m, c_rpt, dacc, h->hacc_dev));
       return SPGEMM_OK;
     };
     const spgemm_status_t ss = run_graph(h, h->gsmall, topo, ptrs, enqueue);

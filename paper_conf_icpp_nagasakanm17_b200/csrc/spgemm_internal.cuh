@@ -831,7 +831,8 @@ cudaError_t launch_scan_and_group(cudaStream_t s, long long m, int64_t* c_rpt, c
                                   uint8_t* grp2, DevAcc* acc, Bounds b, EscSel esc,
                                   long long* tile_ws, int* nlaunch);
 size_t scan_workspace_bytes(long long m);
-cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc);
+// host_acc: pinned host copy of acc written by the kernel at its end (nullptr: none)
+cudaError_t launch_scan_small(cudaStream_t s, long long m, int64_t* c_rpt, DevAcc* acc, DevAcc* host_acc);
 cudaError_t launch_validate(cudaStream_t s, long long m, long long k, long long n, const int64_t* a_rpt,
                             const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int* err);
 cudaError_t launch_partition(cudaStream_t s, long long m, const int64_t* a_rpt, const int32_t* a_col,

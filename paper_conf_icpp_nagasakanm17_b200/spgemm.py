@@ -104,6 +104,10 @@ class Handle:
         self.c_rpt = None
         self.nnz_c = 0
         self.nprod = 0
+        # per-call ctypes objects and entry points, made once (host latency of small multiplies)
+        self._nnz_out, self._nprod_out = ctypes.c_int64(), ctypes.c_int64()
+        self._nnz_ref, self._nprod_ref = ctypes.byref(self._nnz_out), ctypes.byref(self._nprod_out)
+        self._f_sym, self._f_num = lib.spgemm_symbolic, lib.spgemm_numeric
 
     # ----------------------------------------------------------------- options / info
     def set_option(self, name: str, value: int) -> "Handle":
@@ -144,14 +148,12 @@ class Handle:
             raise ValueError(f"shape mismatch: A is {A.m}x{A.n}, B is {B.m}x{B.n}")
         if c_rpt is None:
             c_rpt = self._empty(A.m + 1, torch.int64)
-        nnz = ctypes.c_int64()
-        nprod = ctypes.c_int64()
-        st = load().spgemm_symbolic(self._h, A.m, B.m, B.n, _ptr(A.rpt), _ptr(A.col), _ptr(B.rpt), _ptr(B.col),
-                                    _ptr(c_rpt), ctypes.byref(nnz), ctypes.byref(nprod))
+        st = self._f_sym(self._h, A.m, B.m, B.n, _ptr(A.rpt), _ptr(A.col), _ptr(B.rpt), _ptr(B.col), _ptr(c_rpt),
+                         self._nnz_ref, self._nprod_ref)
         check(st, self._h, "spgemm_symbolic")
         self._A, self._B, self.c_rpt = A, B, c_rpt
-        self.nnz_c, self.nprod = nnz.value, nprod.value
-        return c_rpt, nnz.value, nprod.value
+        self.nnz_c, self.nprod = self._nnz_out.value, self._nprod_out.value
+        return c_rpt, self.nnz_c, self.nprod
 
     def numeric(self, a_val: torch.Tensor, b_val: torch.Tensor, c_col: torch.Tensor, c_val: torch.Tensor) -> None:
         """Phase 2 (PAPER.md:80 steps (6)-(7)), asynchronous on the handle's stream."""
@@ -162,14 +164,18 @@ class Handle:
             raise TypeError(f"unsupported dtype {a_val.dtype}")
         if c_col.dtype != torch.int32 or c_col.numel() != self.nnz_c or c_val.numel() != self.nnz_c:
             raise ValueError("c_col/c_val must hold exactly nnz(C) entries (int32 / value dtype)")
-        st = load().spgemm_numeric(self._h, dt, _ptr(a_val), _ptr(b_val), _ptr(c_col), _ptr(c_val))
+        st = self._f_num(self._h, dt, _ptr(a_val), _ptr(b_val), _ptr(c_col), _ptr(c_val))
         check(st, self._h, "spgemm_numeric")
 
     def multiply(self, A: CsrMatrix, B: CsrMatrix) -> CsrMatrix:
         """C = A * B with C allocated to its exact nnz."""
         c_rpt, nnz, _ = self.symbolic(A, B)
-        c_col = self._empty(nnz, torch.int32)
-        c_val = self._empty(nnz, A.val.dtype)
+        # col and val of C in one allocation of exactly nnz(C) entries each (PAPER.md:80, 282)
+        vs = A.val.element_size()
+        off = (4 * nnz + 15) // 16 * 16
+        buf = self._empty(off + vs * nnz, torch.uint8)
+        c_col = buf[:4 * nnz].view(torch.int32)
+        c_val = buf[off:off + vs * nnz].view(A.val.dtype)
         self.numeric(A.val, B.val, c_col, c_val)
         return CsrMatrix(A.m, B.n, c_rpt, c_col, c_val)
 
