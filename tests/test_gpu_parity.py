@@ -736,6 +736,31 @@ def test_rank_gout_groups(spg, name):
     assert _rank_rows(got[3]) > 0
 
 
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_rank_big_groups_duplicates_unsorted(spg, dtype):
+    """Numeric groups 9-10 (output reduced into C; level 2 in shared memory) and the chunked symbolic
+    count on B rows with duplicate and unsorted columns: equal keys share one rank and are summed
+    (reading R7); integer values, bit-exact."""
+    rng = np.random.default_rng(36)
+    m, k, n = 360, 1 << 16, 1 << 21
+    la = np.where(np.arange(m) % 2 == 0, rng.integers(190, 330, size=m), rng.integers(450, 900, size=m))
+    rows = np.repeat(np.arange(m), la)
+    A = from_coo(m, k, rows, rng.integers(0, k, size=rows.size), rng.integers(-3, 4, rows.size).astype(float),
+                 dedup=False)
+    br = np.repeat(np.arange(k), 24)
+    bc = rng.integers(0, n, size=br.size)
+    dup = rng.random(br.size) < 0.2
+    bc[dup] = bc[np.maximum(np.arange(br.size) - 1, 0)][dup]
+    B = from_coo(k, n, br, bc, rng.integers(-3, 4, br.size).astype(float), dedup=False)
+    r = np.repeat(np.arange(B.m), np.diff(B.rpt))
+    o = np.lexsort((rng.random(r.size), r))
+    B.col[:] = B.col[o]
+    B.val[:] = B.val[o]
+    for opts in ({}, {"rank_big_sym": 2, "rank_big_shared": 2}, {"rank_mid": 1}):
+        got = check(spg, A, B, dtype, exact=True, opts=opts, what=f"dup/unsorted big groups {opts}")
+        assert got[3]["num_rows"][9] > 0 and got[3]["num_rows"][10] > 0, got[3]["num_rows"]
+
+
 def test_rank_acc_big_rows_int_exact(spg):
     A, B = _big_rows(32)
     check(spg, A.with_values("int", 3), B.with_values("int", 4), np.float32, exact=True, what="big rows int")
