@@ -12,8 +12,9 @@ hash count, scan) -> exact allocation of C -> numeric (grouping, accumulate, gat
 
 N GPUs (torchrun, one rank per GPU, NCCL): the rows of C are independent, so the
 SAME matrix is split into n_prod-balanced row blocks (strong scaling): rank 0
-holds A, B = A is broadcast in chunks (NCCL), every rank computes the same split points on its GPU,
-multiplies its zero-copy row block, and the nnz counts are all-gathered (dist.py).  `value` times
+holds A, B = A is broadcast in chunks (NCCL) while rank 0 computes the split points on its GPU
+(then broadcast), every rank multiplies its zero-copy row block, and the nnz counts are all-gathered
+(dist.py).  `value` times
 the per-rank step (the local two-phase SpGEMM), max over ranks; `e2e` adds the host->device copy,
 the broadcast, the partition, the all-gather and the device->host copy of every rank's C block.
 
@@ -301,10 +302,13 @@ def run_ours(args):
     dA0 = P.CsrMatrix.from_host(A, dev, tdt) if rank == 0 else None
     barrier()
     t0 = time.perf_counter()
-    Bd = D.broadcast_csr(dA0, 0, dev, tdt) if world > 1 else dA0
+    if world > 1:  # chunked broadcast with the n_prod split computed on rank 0 meanwhile
+        _, Bd, splits = D.broadcast_and_partition(dA0, None, src=0, device=dev, dtype=tdt, world=world,
+                                                  partition=D.cuda_partition(h), square=True)
+    else:
+        Bd, splits = dA0, D.cuda_partition(h)(dA0, dA0, 1)
     barrier()
     bcast_s = time.perf_counter() - t0
-    splits = D.cuda_partition(h)(Bd, Bd, world)
     r0, r1 = splits[rank], splits[rank + 1]
     mine = D.row_slice(Bd, r0, r1)
 
@@ -452,8 +456,8 @@ def run_ours(args):
                 dA2 = hA.to(dev, non_blocking=True) if rank == 0 else None
             if world > 1:
                 with torch.cuda.stream(stream):
-                    B2 = D.broadcast_csr(dA2, 0, dev, tdt)
-                    sp = D.cuda_partition(h)(B2, B2, world)
+                    _, B2, sp = D.broadcast_and_partition(dA2, None, src=0, device=dev, dtype=tdt, world=world,
+                                                          partition=D.cuda_partition(h), square=True)
             else:
                 B2, sp = dA2, [0, A.m]
             C = h.multiply(D.row_slice(B2, sp[rank], sp[rank + 1]), B2)

@@ -5,8 +5,8 @@ steps are replicating B (and A when it lives on one rank) and exchanging the per
 counts.  One process per GPU (torch.distributed, NCCL over NVLink/NVSwitch):
 
   1. broadcast B (and A) from `src` — the sizes first, then rpt / col / val in 64 MB chunks;
-  2. every rank computes the same n_prod-balanced split points (spgemm_row_partition, on its
-     own GPU — no collective needed, the splits agree by construction);
+  2. the n_prod-balanced split points (spgemm_row_partition) are computed on `src` while the
+     chunks of step 1 are in flight, then broadcast (P+1 integers);
   3. rank p runs the two-phase SpGEMM on rows [s_p, s_{p+1}) of A as a zero-copy slice
      (a_rpt[0] != 0 is allowed by the C ABI);
   4. all_gather of the P nnz counts -> each rank's offset into the global C;
@@ -42,19 +42,24 @@ class ShardResult:
 BCAST_CHUNK_BYTES = 64 << 20  # NCCL broadcast granularity (many in flight; large tensors pipelined)
 
 
-def _bcast_chunked(t: torch.Tensor, src: int, group=None, chunk_bytes: int = BCAST_CHUNK_BYTES) -> None:
+def _bcast_chunked(t: torch.Tensor, src: int, group=None, chunk_bytes: int = BCAST_CHUNK_BYTES, wait: bool = True):
     """Broadcast a contiguous tensor in chunks (asynchronous ops, waited together), so a
-    gigabyte-sized B is pipelined through the collective instead of one monolithic call."""
+    gigabyte-sized B is pipelined through the collective instead of one monolithic call.
+    wait=False returns the pending works (the caller overlaps other work with them)."""
     flat = t.view(-1)
     per = max(1, chunk_bytes // max(1, t.element_size()))
     works = [dist.broadcast(flat[i:i + per], src, group=group, async_op=True) for i in range(0, flat.numel(), per)]
+    if not wait:
+        return works
     for w in works:
         w.wait()
+    return []
 
 
-def broadcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None) -> CsrMatrix:
+def broadcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None, wait: bool = True):
     """Replicate a CSR matrix held by rank `src` on every rank of `group` (sizes first, then
-    rpt / col / val in chunks)."""
+    rpt / col / val in chunks).  wait=False returns (matrix, pending works): the arrays are valid
+    once the works are waited."""
     rank = dist.get_rank(group)
     meta = torch.zeros(3, dtype=torch.int64, device=device)
     if rank == src:
@@ -67,13 +72,38 @@ def broadcast_csr(M: Optional[CsrMatrix], src: int, device, dtype, group=None) -
         rpt = torch.empty(m + 1, dtype=torch.int64, device=device)
         col = torch.empty(nnz, dtype=torch.int32, device=device)
         val = torch.empty(nnz, dtype=dtype, device=device)
+    works = []
     for t in (rpt, col, val):
         if t.numel():
-            _bcast_chunked(t, src, group)
-    return CsrMatrix(m, n, rpt, col, val)
+            works += _bcast_chunked(t, src, group, wait=wait)
+    Md = CsrMatrix(m, n, rpt, col, val)
+    return Md if wait else (Md, works)
 
 
 _bcast_csr = broadcast_csr
+
+
+def broadcast_and_partition(A: Optional[CsrMatrix], B: Optional[CsrMatrix], *, src: int, device, dtype, world: int,
+                            partition: Callable[[CsrMatrix, CsrMatrix, int], list], square: bool = False,
+                            group=None):
+    """Replicate B (and A) from `src` and agree on the n_prod-balanced split points, with the
+    n_prod pass overlapped with the broadcast: `src` holds both matrices, so it computes the split
+    while the chunks are in flight (collective stream) and sends the P+1 points afterwards; the
+    other ranks only receive.  Returns (A, B, splits) on every rank."""
+    rank = dist.get_rank(group)
+    Bd, works = broadcast_csr(B if not square else A, src, device, dtype, group, wait=False)
+    if square:
+        Ad = Bd
+    else:
+        Ad, wa = broadcast_csr(A, src, device, dtype, group, wait=False)
+        works += wa
+    sp = torch.zeros(world + 1, dtype=torch.int64, device=device)
+    if rank == src:  # the local copies are complete on src: no need to wait for the collective
+        sp.copy_(torch.as_tensor([int(x) for x in partition(Ad, Bd, world)], dtype=torch.int64))
+    for w in works:
+        w.wait()
+    dist.broadcast(sp, src, group=group)
+    return Ad, Bd, [int(x) for x in sp.tolist()]
 
 
 def row_slice(A: CsrMatrix, r0: int, r1: int) -> CsrMatrix:
@@ -92,9 +122,8 @@ def distributed_spgemm(A: Optional[CsrMatrix], B: Optional[CsrMatrix], *, device
     broadcast).  partition(A, B, P) -> P+1 split points; local_multiply(A_rows, B) ->
     (CsrMatrix C_rows, nprod).  Returns a ShardResult (and the global rpt when gather_rpt)."""
     rank, world = dist.get_rank(group), dist.get_world_size(group)
-    Bd = _bcast_csr(B if not square else A, src, device, dtype, group)
-    Ad = Bd if square else _bcast_csr(A, src, device, dtype, group)
-    splits = [int(x) for x in partition(Ad, Bd, world)]
+    Ad, Bd, splits = broadcast_and_partition(A, B, src=src, device=device, dtype=dtype, world=world,
+                                             partition=partition, square=square, group=group)
     r0, r1 = splits[rank], splits[rank + 1]
     C, nprod = local_multiply(row_slice(Ad, r0, r1), Bd)
     counts = torch.tensor([C.nnz], dtype=torch.int64, device=device)
