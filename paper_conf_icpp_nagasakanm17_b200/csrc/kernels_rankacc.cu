@@ -273,11 +273,12 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   };
   // level 2 of the blocks with compact index in [c0, c0 + UPPER) (symbolic rows with more
   // non-empty blocks than UPPER take them in chunks; numeric: c0 = 0 and nb <= UPPER)
+  bool chk2 = chk;  // level 2: symbolic rows decide from level 1 (below)
   auto set_fine = [&](int k, int c0) {
     const unsigned d = (unsigned)(k - lo);
     const int b = blk_of(d) - c0;
     const unsigned bit = 1u << (d & 31);
-    if ((NUM || (unsigned)b < (unsigned)UPPER) && (!chk || !(fine[b] & bit))) atomicOr(fine + b, bit);
+    if ((NUM || (unsigned)b < (unsigned)UPPER) && (!chk2 || !(fine[b] & bit))) atomicOr(fine + b, bit);
   };
   int32_t* cc_row = nullptr;
   VT* cv_row = nullptr;
@@ -329,6 +330,11 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   int nb;
   if constexpr (sizeof(P1T) == 4) nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
   else nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
+  // symbolic: nearly one non-empty 32-column block per product (nb >= 7/8 n_prod_i: a graph row)
+  // means level-2 bits are almost all new, so they are set without reading them first
+  if constexpr (!NUM) {
+    if (SPG_RANK_SETCHECK == 2) chk2 = 8LL * nb < 7LL * P;
+  }
   // CTA-uniform; numeric: false only for inconsistent input (the symbolic count bounds nb)
   const bool ok = !NUM || nb <= (int)UPPER;
   auto level2 = [&](int c0) {
