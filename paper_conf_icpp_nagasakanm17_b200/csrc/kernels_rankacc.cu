@@ -319,9 +319,26 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
         if constexpr (NUM) val[u] = sav[e] * __ldg(bv_g + q);
       }
     }
+    int u0 = 0;
+    if constexpr (!NUM) {
+      if (SPG_RANK_SETCHECK == 2) {
+        // symbolic: the first product of every thread sets its level-1 bit after reading it; if
+        // more than 1 in 32 of these found the bit already set the row repeats blocks and keeps
+        // reading, else (a graph row) the rest set their bits unread
+        bool hit = false;
+        if (key[0] >= 0) {
+          const unsigned d = (unsigned)(key[0] - lo);
+          const unsigned bit = 1u << ((d >> 5) & 31);
+          hit = (l1[d >> 10] & bit) != 0;
+          if (!hit) atomicOr(l1 + (d >> 10), bit);
+        }
+        chk = 32 * __syncthreads_count(hit) > TPR;
+        u0 = 1;
+      }
+    }
 #pragma unroll
     for (int u = 0; u < KP; ++u)
-      if (key[u] >= 0) set_l1(key[u]);
+      if (u >= u0 && key[u] >= 0) set_l1(key[u]);
   } else {
     walk([&](int k, VT) { set_l1(k); });
   }
