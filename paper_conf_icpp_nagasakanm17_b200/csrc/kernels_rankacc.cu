@@ -595,11 +595,14 @@ __global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankbig(NumArgs a) {
       const unsigned w = d >> 10, bit = (d >> 5) & 31;
       return (int)p1[w] + __popc(l1[w] & ((1u << bit) - 1u));
     };
+    // set-if-clear only on rows whose columns repeat (n_prod_i > 17/16 nnz_i), as in rank_row
+    const bool chk = SPG_RANK_SETCHECK == 1 ||
+                     (SPG_RANK_SETCHECK == 2 && (a.nprod == nullptr || a.nprod[row] > (long long)cn + (cn >> 4)));
     __syncthreads();
     walk([&](int k, VT) {
       const unsigned d = (unsigned)(k - lo);
       const unsigned bit = 1u << ((d >> 5) & 31);
-      if (!(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
+      if (!chk || !(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
     });
     __syncthreads();
     const int nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
