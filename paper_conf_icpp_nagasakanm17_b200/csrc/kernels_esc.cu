@@ -382,13 +382,13 @@ __global__ __launch_bounds__(TPR, (sizeof(VT) == 8 ? SPG_ESC64_OCC : kEscOcc) / 
   const int Pt = sm->rt.pbase[nr];
   constexpr int KB = KP;  // counters per thread
   {
-    int mx = 0;
+    int c[KB];
+    esc_scan_counts<TPR, KB>(sm->cnt, sm->ws, c);
+    int mx = 0;  // the largest bucket (from the counts the scan read; published by the barrier below)
 #pragma unroll
-    for (int i = 0; i < KB; ++i) mx = max(mx, sm->cnt[sw4(t * KB + i)]);
+    for (int i = 0; i < KB; ++i) mx = max(mx, c[i]);
     mx = __reduce_max_sync(kFull, mx);
     if ((t & 31) == 0 && mx > kEscSkew) atomicMax(&sm->smax, mx);
-    int c[KB];
-    esc_scan_counts<TPR, KB>(sm->cnt, sm->ws, c);  // (its barriers publish smax)
   }
   __syncthreads();
   if (sm->smax > kEscSkew) {
