@@ -8,7 +8,7 @@
 // kernels on rows of a few hundred products.
 //
 //   k_sym_batch  step (3): every product's column is inserted into its row's
-//                hash table in shared memory — Alg. 5 verbatim (key*HASH_SCAL mod t_size,
+//                hash table in shared memory — Alg. 5 (multiplicative hash of the key into t_size slots,
 //                linear probing, atomicCAS from -1), t_size = 4*next_pow2(n_prod_i) (2* for the largest group) — and
 //                nnz_i = the number of successful inserts.
 //   k_num_esc    step (7): the paper accumulates into a hash table, gathers
