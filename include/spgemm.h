@@ -178,7 +178,7 @@ typedef enum {
                                        clear + prefix costs more than the row).  Default 500,
                                        0 = no limit */
     SPGEMM_OPT_RANK_L1_PCT_SYM = 20,/* same for the symbolic rank-count kernels, B = the group's
-                                       n_prod bound.  Default 150, 0 = no limit */
+                                       n_prod bound.  Default 100, 0 = no limit */
     SPGEMM_OPT_BATCH = 21,          /* batched graph-row kernels, bit mask:
                                        1 = symbolic groups 2-9 by the paper hash (Alg. 5), R rows
                                        of one group per CTA with their products flattened;

@@ -107,7 +107,9 @@ struct spgemm_ctx {
   // R-MAT s22 (4097 words), rank vs paper hash + bucket sort: numeric group 4 (bound 256) 11.6 vs
   // 4.1 ms, group 5 (512) 13.5 vs 9.0, group 6 (1024) 14.6 vs 17.8; symbolic group 6 (2048) 6.7
   // vs 4.5, group 7 (4096) 3.6 vs 4.6
-  long long rank_l1_pct = 500, rank_l1_pct_sym = 150;
+  // (symbolic 100 since the multiplicative hash's top-bit slots: R-MAT s22 symbolic group 7 hash 2.94 vs
+  // rank count 3.33 ms; s20 group 5 0.71 vs 0.73; other configs unchanged)
+  long long rank_l1_pct = 500, rank_l1_pct_sym = 100;
   int tiny = 1;          // groups 0-1: thread-per-row register tables (kernels_tiny.cu)
   int small_opt = 1;     // small matrices (m <= kSmallRows): one-launch phases, no grouping (kernels_tiny.cu)
   // warp-per-row register sort (kernels_wsort.cu): bit 1 symbolic, bit 2 numeric.  Off by default:
