@@ -73,40 +73,53 @@ __device__ __forceinline__ int cta_scan32(int v, int* total, int* ws32) {
 
 __device__ __forceinline__ int popc4(uint4 x) { return __popc(x.x) + __popc(x.y) + __popc(x.z) + __popc(x.w); }
 
+#ifndef SPG_L1_SWIZZLE
+#define SPG_L1_SWIZZLE 1
+#endif
+// Level-1 word w (and its prefix) lives at l1sw(w): bits 2-4 XOR bits 5-7.  The bank of a word is
+// bits 0-4 of its index, i.e. bits 10-14 of the column offset, which are biased on R-MAT (a 1 with
+// p = 0.4 per bit); XOR with the next bits evens the banks out.  Groups of 4 words stay together
+// (uint4 sweeps); arrays are padded to 32 words.
+__device__ __forceinline__ int l1sw(int w) { return SPG_L1_SWIZZLE ? w ^ (((w >> 5) & 7) << 2) : w; }
+__host__ __device__ constexpr int l1_pad(int w) { return SPG_L1_SWIZZLE ? (w + 31) & ~31 : (w + 3) & ~3; }
+
 // Exclusive prefix popcount of words[0..W) (W rounded up to 4 words, the tail zero) into pre
-// (u16, may be null); returns the total.  One contiguous run of uint4 per thread.
-template <int TPR>
+// (u16, may be null); returns the total.  One contiguous run of uint4 per thread.  SW: words and
+// pre are laid out by l1sw (level 1).
+template <int TPR, bool SW = false>
 __device__ __forceinline__ int prefix_popc(const unsigned* words, int W, uint16_t* pre, int* ws32) {
   const int W4 = (W + 3) >> 2;
   const int per = (W4 + TPR - 1) / TPR;
   const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
   const uint4* w4 = reinterpret_cast<const uint4*>(words);
+  auto ph = [](int v) { return SW ? l1sw(4 * v) >> 2 : v; };
   int loc = 0;
-  for (int v = v0; v < v1; ++v) loc += popc4(w4[v]);
+  for (int v = v0; v < v1; ++v) loc += popc4(w4[ph(v)]);
   int total;
   int run = cta_scan32<TPR>(loc, &total, ws32);
   if (pre) {
     for (int v = v0; v < v1; ++v) {
-      const uint4 x = w4[v];
+      const uint4 x = w4[ph(v)];
       ushort4 o;
       o.x = (unsigned short)run; run += __popc(x.x);
       o.y = (unsigned short)run; run += __popc(x.y);
       o.z = (unsigned short)run; run += __popc(x.z);
       o.w = (unsigned short)run; run += __popc(x.w);
-      reinterpret_cast<ushort4*>(pre)[v] = o;
+      reinterpret_cast<ushort4*>(pre)[ph(v)] = o;
     }
   }
   return total;
 }
 
 // u32 variant (prefix values above 65535; `global`: the words live in a global slab, read via L2)
-template <int TPR>
+template <int TPR, bool SW = false>
 __device__ __forceinline__ int prefix_popc32(const unsigned* words, int W, unsigned* pre, int* ws32, bool global) {
   const int W4 = (W + 3) >> 2;
   const int per = (W4 + TPR - 1) / TPR;
   const int v0 = min(W4, (int)threadIdx.x * per), v1 = min(W4, v0 + per);
   const uint4* w4 = reinterpret_cast<const uint4*>(words);
-  auto ld = [&](int v) { return global ? __ldcg(w4 + v) : w4[v]; };
+  auto ph = [](int v) { return SW ? l1sw(4 * v) >> 2 : v; };
+  auto ld = [&](int v) { return global ? __ldcg(w4 + ph(v)) : w4[ph(v)]; };
   int loc = 0;
   for (int v = v0; v < v1; ++v) loc += popc4(ld(v));
   int total;
@@ -118,7 +131,7 @@ __device__ __forceinline__ int prefix_popc32(const unsigned* words, int W, unsig
     o.y = (unsigned)run; run += __popc(x.y);
     o.z = (unsigned)run; run += __popc(x.z);
     o.w = (unsigned)run; run += __popc(x.w);
-    reinterpret_cast<uint4*>(pre)[v] = o;
+    reinterpret_cast<uint4*>(pre)[ph(v)] = o;
   }
   return total;
 }
@@ -148,10 +161,10 @@ struct RankLayout {
   static constexpr int kFine = kKeys + (kOwnOut ? align16((int)UPPER * 4) : 0);
   static constexpr int kBstart = kFine + align16((int)UPPER * 4);
   static constexpr int kL1 = kBstart + align16((KP * TPR / 32 + 1) * 4);
-  static __host__ __device__ constexpr int pre2(int l1w) { return kL1 + align16(l1w * 4); }
+  static __host__ __device__ constexpr int pre2(int l1w) { return kL1 + align16(l1_pad(l1w) * 4); }
   static __host__ __device__ constexpr int p1(int l1w) { return pre2(l1w) + (NUM ? align16((int)UPPER * 2) : 0); }
   using P1T = std::conditional_t<(!NUM && UPPER > 16384), unsigned, uint16_t>;
-  static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1w * (int)sizeof(P1T)); }
+  static __host__ __device__ constexpr int bytes(int l1w) { return p1(l1w) + align16(l1_pad(l1w) * (int)sizeof(P1T)); }
 };
 
 // Per-group launch shape of the rank kernels (independent of the hash groups' Table-I shapes):
@@ -172,7 +185,7 @@ constexpr RankCfg kRankNum[] = {{0, 0, 0},   {0, 0, 0},    {0, 0, 0},    {64, 4,
 // 0.53/0.69 ms); MC 4 measured slower than 2 for groups 5-8
 constexpr RankCfg kRankSym[] = {{0, 0, 0},    {0, 0, 0},    {0, 0, 0},    {64, 4, 2},   {64, 8, 2},
                                 {64, 16, 2},  {128, 16, 2}, {256, 16, 2}, {512, 16, 2}, {1024, 16, 2}};
-__host__ __device__ constexpr int rankbig_l1pad_h(int l1w) { return (l1w + 3) & ~3; }
+__host__ __device__ constexpr int rankbig_l1pad_h(int l1w) { return ((l1w + 31) & ~31); }
 
 // Adapters so rank_row reads both argument structs the same way.
 struct NumView : NumArgs {
@@ -214,7 +227,7 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   const int2 rr = __ldg(a.rlohi + row);
   const int lo = rr.x;
   const int W1 = rr.y >= rr.x ? (int)(((unsigned)(rr.y - rr.x)) >> 10) + 1 : 0;  // CTA-uniform
-  clear_words<TPR>(l1, W1);
+  clear_words<TPR>(l1, l1_pad(W1));
 
   // (i) metadata: thread t owns A non-zeros t*MC .. t*MC+MC-1
   int lens[MC];
@@ -265,10 +278,12 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   auto set_l1 = [&](int k) {
     const unsigned d = (unsigned)(k - lo);
     const unsigned bit = 1u << ((d >> 5) & 31);
-    if (!chk || !(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
+    const int w = l1sw((int)(d >> 10));
+    if (!chk || !(l1[w] & bit)) atomicOr(l1 + w, bit);
   };
   auto blk_of = [&](unsigned d) {
-    const unsigned w = d >> 10, bit = (d >> 5) & 31;
+    const int w = l1sw((int)(d >> 10));
+    const unsigned bit = (d >> 5) & 31;
     return (int)p1[w] + __popc(l1[w] & ((1u << bit) - 1u));
   };
   // level 2 of the blocks with compact index in [c0, c0 + UPPER) (symbolic rows with more
@@ -329,8 +344,9 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
         if (key[0] >= 0) {
           const unsigned d = (unsigned)(key[0] - lo);
           const unsigned bit = 1u << ((d >> 5) & 31);
-          hit = (l1[d >> 10] & bit) != 0;
-          if (!hit) atomicOr(l1 + (d >> 10), bit);
+          const int w = l1sw((int)(d >> 10));
+          hit = (l1[w] & bit) != 0;
+          if (!hit) atomicOr(l1 + w, bit);
         }
         chk = 32 * __syncthreads_count(hit) > TPR;
         u0 = 1;
@@ -345,8 +361,8 @@ __device__ __forceinline__ void rank_row(const Args& a, int row, unsigned char* 
   __syncthreads();
   // (iii) compact index of the non-empty 32-column blocks
   int nb;
-  if constexpr (sizeof(P1T) == 4) nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
-  else nb = prefix_popc<TPR>(l1, W1, p1, ws32[1]);
+  if constexpr (sizeof(P1T) == 4) nb = prefix_popc32<TPR, true>(l1, W1, p1, ws32[1], false);
+  else nb = prefix_popc<TPR, true>(l1, W1, p1, ws32[1]);
   // symbolic: nearly one non-empty 32-column block per product (nb >= 7/8 n_prod_i: a graph row)
   // means level-2 bits are almost all new, so they are set without reading them first
   if constexpr (!NUM) {
@@ -585,14 +601,15 @@ __global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankbig(NumArgs a) {
     const int cn = (int)(a.c_rpt[row + 1] - c0);
     int32_t* __restrict__ cc = a.c_col + c0;
     VT* __restrict__ cv = static_cast<VT*>(a.c_val) + c0;
-    clear_words<TPR>(l1, W1);
+    clear_words<TPR>(l1, l1_pad(W1));
     for (int r = t; r < cn; r += TPR) cv[r] = VT(0);
     auto walk = [&](auto&& f) {
       for_each_product_block<true, false, VT, TPR>(a.a_rpt, a.a_col, av_g, a.b_rpt, a.b_col, bv_g, true, row, t, bf,
                                                    ws64, f, NoStopR{});
     };
     auto blk_of = [&](unsigned d) {
-      const unsigned w = d >> 10, bit = (d >> 5) & 31;
+      const int w = l1sw((int)(d >> 10));
+      const unsigned bit = (d >> 5) & 31;
       return (int)p1[w] + __popc(l1[w] & ((1u << bit) - 1u));
     };
     // set-if-clear only on rows whose columns repeat (n_prod_i > 17/16 nnz_i), as in rank_row
@@ -602,10 +619,11 @@ __global__ __launch_bounds__(TPR, 1024 / TPR) void k_num_rankbig(NumArgs a) {
     walk([&](int k, VT) {
       const unsigned d = (unsigned)(k - lo);
       const unsigned bit = 1u << ((d >> 5) & 31);
-      if (!chk || !(l1[d >> 10] & bit)) atomicOr(l1 + (d >> 10), bit);
+      const int w = l1sw((int)(d >> 10));
+      if (!chk || !(l1[w] & bit)) atomicOr(l1 + w, bit);
     });
     __syncthreads();
-    const int nb = prefix_popc32<TPR>(l1, W1, p1, ws32[1], false);
+    const int nb = prefix_popc32<TPR, true>(l1, W1, p1, ws32[1], false);
     const bool ok = nb <= (SH ? SL2 : (int)a.slab_T);  // CTA-uniform; false only for inconsistent input
     if (ok) {
       uint4* f4 = reinterpret_cast<uint4*>(fine);
