@@ -220,6 +220,10 @@ typedef enum {
     SPGEMM_OPT_RANK_GOUT = 29,      /* 1: numeric rank groups 3-8 reduce values straight into the
                                        zeroed row of C at their rank instead of a shared-memory
                                        row (less shared memory per CTA).  Default 0 */
+    SPGEMM_OPT_RANK_BIG_MAX = 31,   /* numeric rows above the CTA groups (groups 10, 11, 12: up to
+                                       24576 / 49152 / 98304 entries): the first v groups take the
+                                       one-CTA-per-row rank-big kernel, the others the DSMEM cluster
+                                       tables of 2/4/8 CTAs.  Default 3 */
     SPGEMM_OPT_SMALL = 24           /* 1 (default): matrices of <= 65536 rows whose rows all have
                                        n_prod_i <= 32 run each phase as one thread-per-row launch
                                        (register tables, no grouping, one host sync); otherwise,

@@ -27,7 +27,7 @@ OPTIONS = {
     "validate": 4, "lanes": 5, "workspace_budget": 6, "timing": 7, "long_row": 8, "range_hash": 9,
     "cluster": 10, "cluster_fill_limit": 11, "flat": 12, "graphs": 13, "range_warp": 14,
     "range_min_nprod": 15, "bitmap_rank": 16, "rank_acc": 17, "tiny": 18, "rank_l1_pct": 19, "rank_l1_pct_sym": 20,
-    "batch": 21, "esc_pct": 22, "esc_groups": 23, "small": 24, "wsort": 25, "rank_big_sym": 26, "rank_big_shared": 27, "rank_mid": 28, "rank_gout": 29,
+    "batch": 21, "esc_pct": 22, "esc_groups": 23, "small": 24, "wsort": 25, "rank_big_sym": 26, "rank_big_shared": 27, "rank_mid": 28, "rank_gout": 29, "rank_big_max": 31,
 }
 
 # spgemm_kernel_t (include/spgemm.h): kernel family that ran each group

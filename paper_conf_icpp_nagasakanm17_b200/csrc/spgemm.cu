@@ -125,7 +125,8 @@ struct spgemm_ctx {
   // (R-MAT s22 6.87 -> 5.54 ms); 1 = persistent rank-big kernel with level 2 in shared memory
   // (6.32 ms); 0 = one 1024-thread CTA per row, the row in shared memory
   int rank_mid = 2;
-  int rank_gout = 0;  // numeric rank groups 3-8 with the output reduced into C (no vals/keys arrays)  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
+  int rank_gout = 0;
+  int rank_big_max = 3;  // numeric big groups 10..10+rank_big_max-1 on the rank-big kernel, the rest on clusters  // numeric rank groups 3-8 with the output reduced into C (no vals/keys arrays)  // numeric group 10 rank-big rows: level 2 in shared memory (if it fits)
   bool small = false;    // the last symbolic call took the small-matrix path
   std::vector<long long> small_miss;  // inputs whose last small-path attempt overflowed (skip it)
   // batched graph-row kernels (kernels_esc.cu): bit 1 symbolic groups 2-9 (off by default: R-MAT s22
@@ -646,6 +647,9 @@ spgemm_status_t spgemm_set_option(spgemm_handle_t h, spgemm_option_t opt, int64_
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_SHARED must be 0, 1 or 2");
       h->rank_big_shared = (int)v; break;
     case SPGEMM_OPT_RANK_GOUT: h->rank_gout = v ? 1 : 0; break;
+    case SPGEMM_OPT_RANK_BIG_MAX:
+      if (v < 0 || v > 3) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_BIG_MAX must be 0..3");
+      h->rank_big_max = (int)v; break;
     case SPGEMM_OPT_RANK_MID:
       if (v < 0 || v > 2) return fail(h, SPGEMM_ERR_INVALID_ARG, "RANK_MID must be 0, 1 or 2");
       h->rank_mid = (int)v; break;
@@ -1124,10 +1128,12 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
     const bool mid_rank = h->rank_mid == 1 && h->snap2.num_rows[kNumCluster - 1] > 0 && rank_acc_on(kNumCluster - 1) &&
                           kNumGroups[kNumCluster - 1].upper <= kRankMidSharedL2 &&
                           rankbig_smem_bytes(fp64, l1w_rank, 2) <= kSmemLimit / 2;
+    // big groups c < rank_big_max take the rank-big kernel, the others the DSMEM cluster tables
+    auto big_rank_c = [&](int c) { return big_rank && c < h->rank_big_max; };
     for (int c = 0; c < 3; ++c) {
       const long long rows_c = (long long)h->snap2.num_rows[kNumCluster + c];
       if (rows_c == 0) continue;
-      if (big_rank) {
+      if (big_rank_c(c)) {
         bstride[c] = (kNumGroups[kNumCluster + c].upper * 8 + 16 + 255) & ~255LL;
         bgrid[c] = std::min<long long>(rows_c, h->num_sms);
         btotal += bgrid[c] * bstride[c];
@@ -1138,8 +1144,8 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
       ccount[c] = std::min<long long>(nc, rows_c);
       ctotal += ccount[c];
     }
-    if (ctotal > 0) ALLOC(h->num_slab_c, (size_t)(ctotal * cstride));
-    if (btotal > 0) ALLOC(h->num_slab_c, (size_t)btotal);
+    // one slab buffer: cluster regions first, rank-big regions after them
+    if (ctotal > 0 || btotal > 0) ALLOC(h->num_slab_c, (size_t)(ctotal * cstride + btotal));
     const long long n_glob = (long long)h->snap2.num_rows[kNumGlobal];
     int glob_grid = 0;
     if (n_glob > 0) {
@@ -1160,7 +1166,7 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
                                    na.priv_ok, h->use_streams, h->timing, h->m, h->n, h->nnzc, (long long)group_events(h),
                                    h->snap1.range_rmax, (long long)na.l1_words, (long long)h->rank_acc, (long long)h->tiny,
                                    (long long)low_compression, h->rank_l1_pct, (long long)h->bitmap_rank,
-                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)mid_rank, (long long)h->rank_mid, (long long)h->rank_gout, (long long)h->snap2.max_nnz,
+                                   (long long)h->num_min_group, (long long)big_rank, (long long)h->rank_big_shared, (long long)mid_rank, (long long)h->rank_mid, (long long)h->rank_gout, (long long)h->rank_big_max, (long long)h->snap2.max_nnz,
                                    na.slab_T, na.slab_stride, cstride, (long long)na.bitmap_words, (long long)h->wsort};
     for (int g = 0; g < kMaxGroups; ++g) topo.push_back((long long)h->snap2.num_rows[g]);
     const std::vector<long long> ptrs = {(long long)a_val, (long long)b_val, (long long)c_col, (long long)c_val,
@@ -1217,14 +1223,14 @@ spgemm_status_t spgemm_numeric(spgemm_handle_t h, spgemm_dtype_t dt, const void*
             CK(cudaMalloc(&gc.prof, sizeof(unsigned long long) * 4 * rows));
             CK(cudaMemset(gc.prof, 0, sizeof(unsigned long long) * 4 * rows));
           }
-          if (big_rank && c == 0 && h->rank_big_shared == 2 && rankout_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit) {
+          if (big_rank_c(c) && c == 0 && h->rank_big_shared == 2 && rankout_smem_bytes(g, fp64, l1w_rank) <= kSmemLimit) {
             // group 10: products in registers, output reduced into C, one 1024-thread CTA per row
             NumArgs ro = ga;
             ro.l1_words = l1w_rank;
             CK(launch_numeric_rankout(st, g, fp64, ro));
             h->gkind[1][g] = SPGEMM_KERNEL_RANK;
-          } else if (big_rank) {
-            long long boff = 0;
+          } else if (big_rank_c(c)) {
+            long long boff = ctotal * cstride;
             for (int q = 0; q < c; ++q) boff += bgrid[q] * bstride[q];
             gc.slab = static_cast<unsigned char*>(h->num_slab_c.p) + boff;
             gc.slab_stride = bstride[c];

@@ -667,6 +667,9 @@ def test_rank_acc_big_rows(spg, dtype):
     check(spg, A, B, dtype, opts={"rank_big_shared": 0}, what="big rows rank, level 2 in global memory")
     check(spg, A, B, dtype, opts={"rank_big_shared": 2}, what="big rows rank, group 10 in registers, output in C")
     check(spg, A, B, dtype, opts={"rank_mid": 0}, what="big rows rank, group 9 one CTA per row")
+    for mx in (0, 1, 2):  # groups >= 10 + mx on the DSMEM cluster tables, the rest rank-big (one slab)
+        got = check(spg, A, B, dtype, opts={"rank_big_max": mx}, what=f"big rows rank_big_max={mx}")
+        assert all(got[3]["num_kernel"][10 + c] in (0, 4 if c >= mx else 6) for c in range(3)), got[3]["num_kernel"]
     check(spg, A, B, dtype, opts={"rank_acc": 0}, what="big rows cluster")
 
 
