@@ -80,7 +80,8 @@ __device__ __forceinline__ void brow_warp(const int32_t* __restrict__ b_col, lon
 
 __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, const int64_t* __restrict__ b_rpt,
                                                                const int32_t* __restrict__ b_col,
-                                                               int2* __restrict__ bmm, int* __restrict__ unsorted,
+                                                               int2* __restrict__ bmm, int4* __restrict__ binfo,
+                                                               int* __restrict__ unsorted,
                                                                int32_t* __restrict__ defer, int* __restrict__ ndefer) {
   const int glog = setup_glog(b_rpt, k);
   const int G = 1 << glog, lane = threadIdx.x & 31, gl = lane & (G - 1);
@@ -142,7 +143,10 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, cons
       bad |= pbad && lane == src;
       if (lane == src) { mn = pmn; mx = pmx; }
     }
-    if (row < k && gl == 0 && !(defer && is_long && b1 - b0 > kDeferLen)) bmm[row] = make_int2(mn, mx);
+    if (row < k && gl == 0 && !(defer && is_long && b1 - b0 > kDeferLen)) {
+      bmm[row] = make_int2(mn, mx);
+      if (binfo) binfo[row] = make_int4(mn, mx, (int)(b1 - b0), 0);
+    }
   }
   if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(unsorted, 1);
 }
@@ -150,7 +154,8 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax(long long k, cons
 // Deferred long B rows: one warp per row.
 __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax_long(const int64_t* __restrict__ b_rpt,
                                                                     const int32_t* __restrict__ b_col,
-                                                                    int2* __restrict__ bmm, int* __restrict__ unsorted,
+                                                                    int2* __restrict__ bmm, int4* __restrict__ binfo,
+                                                                    int* __restrict__ unsorted,
                                                                     const int32_t* __restrict__ defer,
                                                                     const int* __restrict__ ndefer) {
   const int lane = threadIdx.x & 31;
@@ -160,9 +165,11 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax_long(const int64_
     const int row = defer[i];
     int mn, mx;
     bool bad;
-    brow_warp(b_col, __ldg(b_rpt + row), __ldg(b_rpt + row + 1), lane, mn, mx, bad);
+    const long long r0 = __ldg(b_rpt + row), r1 = __ldg(b_rpt + row + 1);
+    brow_warp(b_col, r0, r1, lane, mn, mx, bad);
     if (lane == 0) {
       bmm[row] = make_int2(mn, mx);
+      if (binfo) binfo[row] = make_int4(mn, mx, (int)(r1 - r0), 0);
       if (bad) atomicOr(unsorted, 1);
     }
   }
@@ -170,8 +177,8 @@ __global__ __launch_bounds__(kSetupThreads) void k_brow_minmax_long(const int64_
 
 // Warp-wide n_prod and column span of A row [s0, s1), 8 entries per lane in flight.
 __device__ __forceinline__ void nprod_warp(const int32_t* __restrict__ a_col, const int64_t* __restrict__ b_rpt,
-                                           const int2* __restrict__ bmm, long long s0, long long s1, int lane,
-                                           long long& np, int& lo, int& hi) {
+                                           const int2* __restrict__ bmm, const int4* __restrict__ binfo,
+                                           long long s0, long long s1, int lane, long long& np, int& lo, int& hi) {
   long long part = 0;
   int plo = INT_MAX, phi = -1;
   for (long long j = s0 + lane; j < s1; j += 8 * 32) {
@@ -181,8 +188,13 @@ __device__ __forceinline__ void nprod_warp(const int32_t* __restrict__ a_col, co
 #pragma unroll
     for (int u = 0; u < 8; ++u)
       if (kk[u] >= 0) {
-        part += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
-        if (bmm) { const int2 r = __ldg(bmm + kk[u]); plo = min(plo, r.x); phi = max(phi, r.y); }
+        if (binfo) {  // one 16-byte gather: span and length of the B row
+          const int4 r = __ldg(binfo + kk[u]);
+          part += r.z; plo = min(plo, r.x); phi = max(phi, r.y);
+        } else {
+          part += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+          if (bmm) { const int2 r = __ldg(bmm + kk[u]); plo = min(plo, r.x); phi = max(phi, r.y); }
+        }
       }
   }
   np = (long long)warp_sum_u64((unsigned long long)part);
@@ -224,7 +236,8 @@ __device__ __forceinline__ int nprod_finish(long long row, long long np, int lo,
 // histogram (CTA-aggregated before the global atomics).
 __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
     long long m, const int64_t* __restrict__ a_rpt, const int32_t* __restrict__ a_col,
-    const int64_t* __restrict__ b_rpt, const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
+    const int64_t* __restrict__ b_rpt, const int2* __restrict__ bmm, const int4* __restrict__ binfo,
+    int64_t* __restrict__ nprod,
     int2* __restrict__ rlohi, uint8_t* __restrict__ grp, int64_t* __restrict__ c_rpt,
     DevAcc* __restrict__ acc, Bounds bd, int32_t* __restrict__ defer, int* __restrict__ ndefer) {
   __shared__ int s_cnt[kMaxGroups];
@@ -257,8 +270,13 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
 #pragma unroll
         for (int u = 0; u < 4; ++u)
           if (kk[u] >= 0) {
-            np += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
-            if (bmm) { const int2 r = __ldg(bmm + kk[u]); lo = min(lo, r.x); hi = max(hi, r.y); }
+            if (binfo) {  // one 16-byte gather: span and length of the B row
+              const int4 r = __ldg(binfo + kk[u]);
+              np += r.z; lo = min(lo, r.x); hi = max(hi, r.y);
+            } else {
+              np += __ldg(b_rpt + kk[u] + 1) - __ldg(b_rpt + kk[u]);
+              if (bmm) { const int2 r = __ldg(bmm + kk[u]); lo = min(lo, r.x); hi = max(hi, r.y); }
+            }
           }
       }
     }
@@ -282,7 +300,7 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
       }
       long long part;
       int plo, phi;
-      nprod_warp(a_col, b_rpt, bmm, s0, s1, lane, part, plo, phi);
+      nprod_warp(a_col, b_rpt, bmm, binfo, s0, s1, lane, part, plo, phi);
       if (lane == src) { np = part; lo = plo; hi = phi; }
     }
     const bool lead = row < m && gl == 0 && !deferred;
@@ -314,7 +332,8 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_group(
 __global__ __launch_bounds__(kSetupThreads) void k_nprod_long(const int64_t* __restrict__ a_rpt,
                                                               const int32_t* __restrict__ a_col,
                                                               const int64_t* __restrict__ b_rpt,
-                                                              const int2* __restrict__ bmm, int64_t* __restrict__ nprod,
+                                                              const int2* __restrict__ bmm,
+                                                              const int4* __restrict__ binfo, int64_t* __restrict__ nprod,
                                                               int2* __restrict__ rlohi, uint8_t* __restrict__ grp,
                                                               int64_t* __restrict__ c_rpt, DevAcc* __restrict__ acc,
                                                               Bounds bd, const int32_t* __restrict__ defer,
@@ -327,7 +346,7 @@ __global__ __launch_bounds__(kSetupThreads) void k_nprod_long(const int64_t* __r
     const int row = defer[i];
     long long np;
     int lo, hi;
-    nprod_warp(a_col, b_rpt, bmm, __ldg(a_rpt + row), __ldg(a_rpt + row + 1), lane, np, lo, hi);
+    nprod_warp(a_col, b_rpt, bmm, binfo, __ldg(a_rpt + row), __ldg(a_rpt + row + 1), lane, np, lo, hi);
     if (lane == 0) {
       int span_max = 0;
       const int g = nprod_finish(row, np, lo, hi, nprod, rlohi, grp, c_rpt, bd, b_ok, span_max);
@@ -623,7 +642,7 @@ __global__ void k_splits(long long m, const int64_t* __restrict__ excl, int npar
 }  // namespace
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
-                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
+                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm, int4* binfo,
                                int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
                                int32_t* defer_a, int32_t* defer_b, int* nlaunch) {
   if (m == 0) return cudaSuccess;
@@ -635,15 +654,16 @@ cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const i
   // deferred long rows (> kDeferLen entries): one warp each, 148 x 4 CTAs of 8 warps
   const unsigned long_grid = 148 * 4;
   if (bmm && k > 0) {
-    k_brow_minmax<<<grid_of(k), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm, &acc->b_unsorted, defer_b,
+    k_brow_minmax<<<grid_of(k), kSetupThreads, 0, s>>>(k, b_rpt, b_col, bmm, binfo, &acc->b_unsorted, defer_b,
                                                        &acc->defer_count[0]);
-    k_brow_minmax_long<<<long_grid, kSetupThreads, 0, s>>>(b_rpt, b_col, bmm, &acc->b_unsorted, defer_b,
+    k_brow_minmax_long<<<long_grid, kSetupThreads, 0, s>>>(b_rpt, b_col, bmm, binfo, &acc->b_unsorted, defer_b,
                                                            &acc->defer_count[0]);
     if (nlaunch) *nlaunch += 2;
   }
-  k_nprod_group<<<grid_of(m), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b,
+  if (!(bmm && k > 0)) binfo = nullptr;  // only k_brow_minmax fills it
+  k_nprod_group<<<grid_of(m), kSetupThreads, 0, s>>>(m, a_rpt, a_col, b_rpt, bmm, binfo, nprod, rlohi, grp, c_rpt, acc, b,
                                                      defer_a, &acc->defer_count[1]);
-  k_nprod_long<<<long_grid, kSetupThreads, 0, s>>>(a_rpt, a_col, b_rpt, bmm, nprod, rlohi, grp, c_rpt, acc, b, defer_a,
+  k_nprod_long<<<long_grid, kSetupThreads, 0, s>>>(a_rpt, a_col, b_rpt, bmm, binfo, nprod, rlohi, grp, c_rpt, acc, b, defer_a,
                                                    &acc->defer_count[1]);
   if (nlaunch) *nlaunch += 2;
   return cudaGetLastError();

@@ -150,6 +150,7 @@ struct spgemm_ctx {
   int64_t* c_rpt = nullptr;
   int vw_log2 = 0;
   Buf defer_b;  // step (1): deferred long B rows (the A list reuses perm1, rewritten after sync 1)
+  Buf binfo;  // step (1): {min col, max col, length} of every B row (one 16-byte gather per A entry)
   Buf nprod, grp1, grp2, perm1, perm2, acc, tiles, overflow, overflow2, slab_sym, bmm, rlohi, num_slab, num_slab_c,
       rbits, bbits;
   bool range_num = false;  // numeric range rows on for the last symbolic call (bitmap allocated, B sorted)
@@ -234,6 +235,7 @@ void release_state(spgemm_handle_t h) {
 void free_all(spgemm_handle_t h) {
   Buf* all[] = {&h->nprod, &h->grp1, &h->grp2, &h->perm1, &h->perm2, &h->acc, &h->tiles, &h->overflow,
                 &h->overflow2, &h->slab_sym, &h->bmm, &h->rlohi, &h->num_slab, &h->num_slab_c, &h->rbits, &h->bbits,
+                &h->binfo,
                 &h->defer_b};
   for (Buf* b : all) buf_free(h, *b);
   release_state(h);
@@ -718,6 +720,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   ALLOC(h->tiles, scan_workspace_bytes(m));
   if (h->range_hash) {
     ALLOC(h->bmm, sizeof(int2) * std::max<int64_t>(k, 1));
+    ALLOC(h->binfo, sizeof(int4) * std::max<int64_t>(k, 1));  // {lo, hi, length} of every B row (step 1)
     ALLOC(h->rlohi, sizeof(int2) * m);
     ALLOC(h->defer_b, sizeof(int32_t) * std::max<int64_t>(k, 1));
   }
@@ -791,6 +794,7 @@ spgemm_status_t spgemm_symbolic(spgemm_handle_t h, int64_t m, int64_t k, int64_t
   {
     int nl = 0;
     CK(launch_nprod_group(h->stream, m, k, a_rpt, a_col, b_rpt, b_col, static_cast<int2*>(h->bmm.p),
+                          static_cast<int4*>(h->binfo.p),
                           static_cast<int64_t*>(h->nprod.p), static_cast<int2*>(h->rlohi.p),
                           static_cast<uint8_t*>(h->grp1.p), c_rpt, dacc, sym_bounds(h),
                           static_cast<int32_t*>(h->perm1.p), static_cast<int32_t*>(h->defer_b.p), &nl));

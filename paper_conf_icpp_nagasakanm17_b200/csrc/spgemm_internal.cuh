@@ -826,7 +826,7 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 
 cudaError_t launch_nprod_group(cudaStream_t s, long long m, long long k, const int64_t* a_rpt,
-                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm,
+                               const int32_t* a_col, const int64_t* b_rpt, const int32_t* b_col, int2* bmm, int4* binfo,
                                int64_t* nprod, int2* rlohi, uint8_t* grp, int64_t* c_rpt, DevAcc* acc, Bounds b,
                                int32_t* defer_a, int32_t* defer_b, int* nlaunch);
 cudaError_t launch_group_stats(cudaStream_t s, long long m, const uint8_t* grp1, const uint8_t* grp2,
